@@ -1,0 +1,165 @@
+"""Pins for the triangulation oracle (Algorithm OPT).
+
+Against: hand-worked examples (tests/golden/*_worked.txt), closed forms for
+n = 3, 4, uniform weights and fans, brute-force enumeration of every
+triangulation for n <= 10 with the Catalan count (golden), and the
+geometric invariances (reflection, rotation) of the problem statement P:149.
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+import bulkgen
+import oracle
+from conftest import read_golden
+
+
+def _parse_worked(name):
+    n, w, expect = None, [], None
+    for row in read_golden(name):
+        if row[0] == "n":
+            n = int(row[1])
+        elif row[0] == "w":
+            w.append((int(row[1]), int(row[2]), int(row[3])))
+        elif row[0] == "expect":
+            expect = (int(row[1]), int(row[2]))
+    c = np.zeros((n, n), dtype=np.int32)
+    for a, b, v in w:
+        c[a, b] = v
+    return c, expect
+
+
+@pytest.mark.parametrize("name", ["pentagon_worked.txt", "hexagon_worked.txt"])
+def test_hand_worked_examples(name):
+    c, (value, count) = _parse_worked(name)
+    assert int(oracle.opt(c)) == value
+    assert int(oracle.opt(c.astype(np.float32))) == value
+    bv, bc = oracle.brute_opt(c)
+    assert (bv, bc) == (value, count)
+
+
+def test_catalan_counts_from_golden():
+    for n, count in ((int(a), int(b)) for a, b in read_golden("catalan_triangulations.txt")):
+        _, cnt = oracle.brute_opt(np.zeros((n, n)))
+        assert cnt == count
+
+
+def test_n3_returns_root_chord_and_zero_with_zero_sides():
+    c = np.zeros((3, 3), dtype=np.int32)
+    assert oracle.opt(c) == 0                      # north_star "n=3 cost 0"
+    c[0, 2] = 17                                   # reading G8: M[1,2] = c[0,2]
+    v, M = oracle.opt(c, return_table=True)
+    assert v == 17 and M[0, 1] == 17 and M[0, 0] == 0 and M[1, 1] == 0
+
+
+def test_n4_closed_form():
+    rng = np.random.default_rng(0)
+    for _ in range(50):
+        c = np.triu(rng.integers(0, 1000, (4, 4)), 2).astype(np.int32)
+        assert oracle.opt(c) == min(c[0, 2], c[1, 3]) + c[0, 3]
+
+
+@pytest.mark.parametrize("n", [5, 8, 12, 16, 40, 64])
+def test_uniform_chord_weights(n):
+    w = 7
+    c = np.zeros((n, n), dtype=np.int32)
+    for a in range(n):
+        for b in range(a + 2, n):
+            if not (a == 0 and b == n - 1):
+                c[a, b] = w
+    assert oracle.opt(c) == (n - 3) * w            # every triangulation has n-3 chords
+    assert oracle.opt(c.astype(np.float32)) == (n - 3) * w
+
+
+@pytest.mark.parametrize("n,v", [(6, 0), (9, 4), (16, 11), (64, 30)])
+def test_fan_from_one_vertex_is_free(n, v):
+    c = np.zeros((n, n), dtype=np.int32)
+    for a in range(n):
+        for b in range(a + 2, n):
+            if not (a == 0 and b == n - 1):
+                c[a, b] = 0 if v in (a, b) else 1
+    assert oracle.opt(c) == 0
+
+
+@pytest.mark.parametrize("n", range(3, 11))
+def test_int32_equals_brute_force(n):
+    for h in range(6 if n < 10 else 2):
+        c = bulkgen.tri_instances(n, [h], seed=100 + n, dtype="int32")[0]
+        bv, cnt = oracle.brute_opt(c)
+        assert oracle.opt(c) == int(bv)
+    assert cnt == [1, 2, 5, 14, 42, 132, 429, 1430][n - 3]
+
+
+@pytest.mark.parametrize("n", range(3, 10))
+def test_fp32_within_rounding_of_exact_brute_force(n):
+    for h in range(4):
+        c = bulkgen.tri_instances(n, [h], seed=200 + n, dtype="float32")[0]
+        bv, _ = oracle.brute_opt(c)
+        v = float(oracle.opt(c))
+        # n-3 chord sums of values < 1: each fp32 add has rel err <= 2^-24
+        assert abs(v - bv) <= (n + 1) * 2.0 ** -24 * max(bv, 1e-30)
+
+
+def test_random_small_weights_many_ties_equal_brute():
+    rng = np.random.default_rng(7)
+    for n in (6, 7, 8):
+        for _ in range(20):
+            c = np.triu(rng.integers(0, 3, (n, n)), 2).astype(np.int32)
+            c[0, n - 1] = rng.integers(0, 3)
+            assert oracle.opt(c) == int(oracle.brute_opt(c)[0])
+
+
+def _reflect(c):
+    n = c.shape[0]
+    r = np.zeros_like(c)
+    for a in range(n):
+        for b in range(a + 1, n):
+            r[n - 1 - b, n - 1 - a] = c[a, b]
+    return r
+
+
+def _rotate(c):
+    # vertex v_x -> v_{x+1 mod n}; chord {a,b} keeps its weight
+    n = c.shape[0]
+    r = np.zeros_like(c)
+    for a in range(n):
+        for b in range(a + 1, n):
+            x, y = (a + 1) % n, (b + 1) % n
+            x, y = min(x, y), max(x, y)
+            r[x, y] = c[a, b]
+    return r
+
+
+@pytest.mark.parametrize("n", [5, 8, 13, 16, 33])
+def test_reflection_and_rotation_invariance(n):
+    c = bulkgen.tri_instances(n, [3], seed=55, dtype="int32")[0]
+    v = oracle.opt(c)
+    assert oracle.opt(_reflect(c)) == v
+    rc = _rotate(c)          # sides stay weight 0 under rotation
+    assert oracle.opt(rc) == v
+    assert oracle.opt(_rotate(rc)) == v
+
+
+def test_table_satisfies_recurrence_identity():
+    # on termination M[i,j] = min_k (M[i,k] + M[k+1,j]) + c[i-1,j]
+    n = 12
+    c = bulkgen.tri_instances(n, [1], seed=9, dtype="int32")[0]
+    _, M = oracle.opt(c, return_table=True)
+    m = lambda i, j: int(M[i - 1, j - 1])
+    for i in range(1, n - 1):
+        assert m(i, i) == 0
+        for j in range(i + 1, n):
+            assert m(i, j) == min(m(i, k) + m(k + 1, j) for k in range(i, j)) + int(c[i - 1, j])
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+def test_bulk_row_and_column_arrangements(dt):
+    n, p = 9, 17
+    row = bulkgen.tri_input(n, p, seed=8, dtype=dt, layout=bulkgen.ROW_WISE)
+    col = bulkgen.tri_input(n, p, seed=8, dtype=dt, layout=bulkgen.COLUMN_WISE)
+    r = oracle.bulk_opt(row, oracle.ROW_WISE)
+    c = oracle.bulk_opt(col, oracle.COLUMN_WISE, nthreads=4)
+    assert np.array_equal(r.view(np.uint32), c.view(np.uint32))
+    for h in range(p):
+        assert r[h] == oracle.opt(row[h])
