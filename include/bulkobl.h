@@ -1,0 +1,178 @@
+/*
+ * bulkobl.h -- C ABI of libbulkobl.so: bulk execution of oblivious sequential
+ * algorithms on NVIDIA B200 (sm_100a).
+ *
+ * Paper: K. Tani, D. Takafuji, K. Nakano, Y. Ito, "Bulk Execution of Oblivious
+ * Algorithms on the Unified Memory Machine, with GPU Implementation",
+ * IPDPS Workshops 2014.  "P:<line>" = line of the paper text.
+ *
+ * The library runs ONE sequential oblivious algorithm on p independent inputs
+ * ("bulk execution").  Two algorithms are provided -- inclusive
+ * prefix sums (Algorithm Prefix-sums) and the minimum-weight convex
+ * polygon triangulation (Algorithm OPT) -- plus the row-wise <->
+ * column-wise layout transpose.
+ *
+ * Conventions for every entry point
+ *   - All data pointers are DEVICE pointers (cudaMalloc / torch CUDA tensors)
+ *     unless the name ends in _host.  The caller owns every buffer; the
+ *     library never allocates, frees or synchronises device memory on the
+ *     device entry points.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *     stream).  Device entry points only enqueue work on it (asynchronous);
+ *     kernel faults surface at the caller's next synchronisation.
+ *   - Return value: BO_OK (0) or a negative bo_status; bulk_last_error()
+ *     returns a thread-local message for the last non-OK status.  No C++
+ *     exception crosses this boundary.  There is no CPU fallback: every
+ *     computation runs in this library's CUDA kernels.
+ *   - Element types are 4-byte: BO_I32 (two's-complement int32, addition
+ *     wraps mod 2^32) or BO_F32 (IEEE binary32, round to nearest).
+ */
+#ifndef BULKOBL_H
+#define BULKOBL_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    BO_OK = 0,
+    BO_EINVAL = -1,        /* bad argument: NULL pointer, size out of range,
+                              overflow of n*p, partial overlap, short workspace */
+    BO_EUNSUPPORTED = -2,  /* a forced variant cannot handle (n, dtype, layout,
+                              alignment); BO_AUTO never returns this          */
+    BO_ECUDA = -3          /* a CUDA launch / copy failed (message has the
+                              cudaGetErrorString text)                         */
+} bo_status;
+
+typedef enum {
+    BO_ROW_WISE = 0,     /* p rows x n columns: b_j[i] at address j*n + i   */
+    BO_COLUMN_WISE = 1   /* n rows x p columns: b_j[i] at address i*p + j   */
+} bo_layout;
+
+typedef enum { BO_I32 = 0, BO_F32 = 1 } bo_dtype;
+
+typedef enum {
+    BO_AUTO = 0,
+    /* prefix sums */
+    BO_PS_ACROSS = 1,      /* column-wise: thread per 4 adjacent instances, 128-bit
+                              coalesced rows, sequential in i (bit-exact)          */
+    BO_PS_WARPSCAN = 2,    /* row-wise: warp per instance, 128-bit lanes + shuffle
+                              scan (fp32 reassociated: not bit-exact)              */
+    BO_PS_FUSED_ROW = 3,   /* row-wise: TMA tiles [128 instances x 32 elements]
+                              through swizzled smem, one thread per instance scans
+                              sequentially (bit-exact), TMA store                  */
+    BO_PS_TRANSPOSED = 4,  /* row-wise: transpose -> BO_PS_ACROSS -> transpose,
+                              needs an n*p*4-byte workspace (bit-exact)            */
+    BO_PS_NAIVE = 5,       /* the paper's GPU kernel: one thread per instance, one
+                              32-bit access per step, any layout      */
+    /* triangulation */
+    BO_TRI_UMM_GLOBAL = 16, /* the paper's Parallel Algorithm OPT: thread per
+                               instance, M in global memory in the same
+                               arrangement as c; workspace
+                               (n-1)^2*p*4 bytes                                  */
+    BO_TRI_SMEM_WARP = 17,  /* warp per instance, M in shared memory, diagonal
+                               wavefront, k split across lanes + shuffle min      */
+    BO_TRI_THREAD_REG = 18, /* thread per instance, M in registers (3 <= n <= 18) */
+    BO_TRI_TILED = 19       /* warp per instance, M in shared memory, 4x4 register
+                               tiles (min-plus blocked product), n <= 64          */
+} bo_variant;
+
+/* ------------------------------------------------------------------------- */
+/* Inclusive prefix sums of p arrays of n elements (Algorithm Prefix-sums,    */
+/* P:95-102; bulk form P:108-118):  dst_j[i] = src_j[0] + ... + src_j[i].     */
+/*   src, dst : device, n*p elements in `layout`; dst == src is the paper's   */
+/*              in-place form; any other overlap is BO_EINVAL.                */
+/*   n >= 0, p >= 0 (n*p == 0 is a no-op); n*p < 2^40.                        */
+/*   fp32 sums are accumulated left to right exactly as P:100 for every       */
+/*   variant except BO_PS_WARPSCAN.                                           */
+/*   workspace: device, >= bulk_prefix_sums_workspace(...) bytes (0 unless    */
+/*   the chosen variant is BO_PS_TRANSPOSED); may be NULL when 0 is needed.   */
+/* ------------------------------------------------------------------------- */
+int bulk_prefix_sums(const void *src, void *dst, int64_t n, int64_t p, int dtype, int layout,
+                     int variant, void *workspace, size_t workspace_bytes, void *stream);
+size_t bulk_prefix_sums_workspace(int64_t n, int64_t p, int dtype, int layout, int variant);
+
+/* ------------------------------------------------------------------------- */
+/* Optimal convex-polygon triangulation of p n-gons (Algorithm OPT, P:174-200;*/
+/* bulk form P:215-237).  out[h] = M_h[1, n-1], where                         */
+/*   M[i,i] = 0,  M[i,j] = min_{i<=k<j} (M[i,k] + M[k+1,j]) + c[i-1, j].      */
+/* That is the minimum total chord weight over all triangulations */
+/* PLUS c[0, n-1] (the root side v0 v_{n-1}, which Algorithm OPT adds; set it */
+/* to 0 to get the pure chord total).  Only entries c[a][b] with b-a >= 2 are */
+/* read.                                                                       */
+/*   c   : device, dense n x n weights per instance.  Row-wise:               */
+/*         c[h*n*n + a*n + b];  column-wise: c[(a*n + b)*p + h]. */
+/*   out : device, p elements of dtype.                                       */
+/*   n >= 3 (n < 3 is BO_EINVAL), p >= 0; n <= 4096.                          */
+/*   int32 weights must satisfy |c| < 2^31 / (2(n-2)) (no overflow); fp32     */
+/*   weights must be finite and >= 0 (results are then bit-identical to the   */
+/*   sequential algorithm: min is exact, every sum keeps its association).    */
+/*   workspace: device, >= bulk_triangulation_workspace(...) bytes (only      */
+/*   BO_TRI_UMM_GLOBAL needs one).                                            */
+/* ------------------------------------------------------------------------- */
+int bulk_triangulation(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout,
+                       int variant, void *workspace, size_t workspace_bytes, void *stream);
+size_t bulk_triangulation_workspace(int64_t n, int64_t p, int dtype, int layout, int variant);
+
+/* ------------------------------------------------------------------------- */
+/* Layout transpose (row-wise <-> column-wise arrangement):        */
+/*   dst[c*rows + r] = src[r*cols + c],  0 <= r < rows, 0 <= c < cols.        */
+/* Row-wise [p][n] -> column-wise [n][p] is (rows=p, cols=n); the reverse is  */
+/* (rows=n, cols=p).  elem_bytes must be 4.  Out of place: src and dst must   */
+/* not overlap.  TMA-tiled when cols%4 == 0, rows%4 == 0 and both pointers    */
+/* are 16-byte aligned; otherwise a padded shared-memory tile kernel.         */
+/* ------------------------------------------------------------------------- */
+int bulk_transpose(const void *src, void *dst, int64_t rows, int64_t cols, size_t elem_bytes,
+                   void *stream);
+
+/* ------------------------------------------------------------------------- */
+/* End-to-end entry points on HOST buffers (pinned memory recommended).       */
+/* The host->device copy, the computation and the device->host copy are       */
+/* pipelined in chunks of instances over two internal streams; the call       */
+/* returns after the result is in h_dst (it synchronises).  d_buf is a device */
+/* buffer of at least n*p*4 bytes (prefix) / n*n*p*4 + p*4 bytes (OPT) plus   */
+/* the variant's workspace; h_dst may equal h_src (prefix).                   */
+/* ------------------------------------------------------------------------- */
+int bulk_prefix_sums_host(const void *h_src, void *h_dst, int64_t n, int64_t p, int dtype,
+                          int layout, int variant, void *d_buf, size_t d_bytes, void *stream);
+int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, int dtype,
+                            int layout, int variant, void *d_buf, size_t d_bytes, void *stream);
+
+/* ------------------------------------------------------------------------- */
+/* Synthetic inputs, generated on the device by the counter-based generator  */
+/* documented in bulkgen/__init__.py (same bits on host and device):         */
+/*   u = mix64(seed*K_SEED + h*K_H + e*K_E), h = GLOBAL instance id h0+local. */
+/* kind: 0 uniform, 1 ones, 2 arange, 3 smallint (prefix only).               */
+/* ------------------------------------------------------------------------- */
+int bulk_generate_prefix(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype,
+                         int layout, int kind, void *stream);
+int bulk_generate_tri(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype,
+                      int layout, void *stream);
+
+/* Order-independent checksum of a result (values: [p][n] row-wise, [n][p]   */
+/* column-wise; n = 1 for per-instance results):                             */
+/*   *acc += sum_{h,e} mix64(bits(v)*K_SEED + (h0+h)*K_H + e*K_E)  mod 2^64.  */
+/* acc is a DEVICE uint64 the caller zeroes.                                 */
+int bulk_checksum(const void *values, int64_t n, int64_t p, int64_t h0, int layout,
+                  uint64_t *acc, void *stream);
+
+/* ------------------------------------------------------------------------- */
+/* Introspection.                                                             */
+/* ------------------------------------------------------------------------- */
+const char *bulk_last_error(void);       /* thread-local message, "" if none     */
+/* Variant BO_AUTO resolves to for these arguments (or the forced one).       */
+int bulk_prefix_sums_variant(int64_t n, int64_t p, int dtype, int layout, int variant,
+                             const void *src, const void *dst);
+int bulk_triangulation_variant(int64_t n, int64_t p, int dtype, int layout, int variant);
+/* Number of CUDA kernels this library has launched in this process.         */
+uint64_t bulk_launch_count(void);
+/* Library version string. */
+const char *bulk_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BULKOBL_H */

@@ -1,0 +1,265 @@
+"""paper_conf_ipps_tanitni14_b200 -- Python binding of libbulkobl.so.
+
+Bulk execution of oblivious sequential algorithms on B200 (Tani, Takafuji,
+Nakano, Ito, IPDPS-W 2014): inclusive prefix sums (Algorithm Prefix-sums,
+P:95-102), optimal convex-polygon triangulation (Algorithm OPT)
+and the row-wise <-> column-wise transpose, each over p
+independent instances.
+
+This module only marshals arguments: torch supplies device memory and the
+current CUDA stream, every step of the computation runs in the CUDA kernels
+of libbulkobl.so (include/bulkobl.h).  There is no CPU fallback: if the
+library is missing or a call fails, a BulkError is raised.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libbulkobl.so")
+
+ROW_WISE, COLUMN_WISE = 0, 1
+I32, F32 = 0, 1
+AUTO = 0
+PS_ACROSS, PS_WARPSCAN, PS_FUSED_ROW, PS_TRANSPOSED, PS_NAIVE = 1, 2, 3, 4, 5
+TRI_UMM_GLOBAL, TRI_SMEM_WARP, TRI_THREAD_REG, TRI_TILED = 16, 17, 18, 19
+VARIANT_NAMES = {
+    AUTO: "auto", PS_ACROSS: "across", PS_WARPSCAN: "warpscan", PS_FUSED_ROW: "fused_row",
+    PS_TRANSPOSED: "transposed", PS_NAIVE: "naive", TRI_UMM_GLOBAL: "umm_global",
+    TRI_SMEM_WARP: "smem_warp", TRI_THREAD_REG: "thread_reg", TRI_TILED: "tiled",
+}
+KINDS = {"uniform": 0, "ones": 1, "arange": 2, "smallint": 3}
+
+
+class BulkError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"bulkobl status {status}: {msg}")
+        self.status = status
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libbulkobl.so (built in-tree by __graft_entry__.build())."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run `python __graft_entry__.py build` "
+                              "(there is no CPU fallback)")
+        L = ctypes.CDLL(LIB_PATH)
+        i64, vp, i32, sz, u64 = ctypes.c_int64, ctypes.c_void_p, ctypes.c_int, ctypes.c_size_t, ctypes.c_uint64
+        sig = {
+            "bulk_prefix_sums": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
+            "bulk_prefix_sums_workspace": ([i64, i64, i32, i32, i32], sz),
+            "bulk_triangulation": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
+            "bulk_triangulation_workspace": ([i64, i64, i32, i32, i32], sz),
+            "bulk_transpose": ([vp, vp, i64, i64, sz, vp], i32),
+            "bulk_prefix_sums_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
+            "bulk_triangulation_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
+            "bulk_generate_prefix": ([vp, i64, i64, i64, u64, i32, i32, i32, vp], i32),
+            "bulk_generate_tri": ([vp, i64, i64, i64, u64, i32, i32, vp], i32),
+            "bulk_checksum": ([vp, i64, i64, i64, i32, vp, vp], i32),
+            "bulk_last_error": ([], ctypes.c_char_p),
+            "bulk_prefix_sums_variant": ([i64, i64, i32, i32, i32, vp, vp], i32),
+            "bulk_triangulation_variant": ([i64, i64, i32, i32, i32], i32),
+            "bulk_launch_count": ([], u64),
+            "bulk_version": ([], ctypes.c_char_p),
+        }
+        for name, (args, res) in sig.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = res
+        _lib = L
+    return _lib
+
+
+def _check(rc: int):
+    if rc != 0:
+        raise BulkError(rc, lib().bulk_last_error().decode())
+
+
+def _dtype_code(t: torch.Tensor) -> int:
+    if t.dtype == torch.int32:
+        return I32
+    if t.dtype == torch.float32:
+        return F32
+    raise TypeError(f"bulkobl supports int32 and float32, got {t.dtype}")
+
+
+def _stream(stream=None) -> int:
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return s.cuda_stream
+
+
+def _need_cuda(*ts):
+    for t in ts:
+        if not t.is_cuda:
+            raise ValueError("device entry points need CUDA tensors (use *_host for host buffers)")
+        if not t.is_contiguous():
+            raise ValueError("tensors must be contiguous")
+
+
+def _shape_np(t: torch.Tensor, layout: int):
+    if t.dim() != 2:
+        raise ValueError("prefix sums take a 2-D tensor: [p, n] row-wise or [n, p] column-wise")
+    return (t.shape[1], t.shape[0]) if layout == ROW_WISE else (t.shape[0], t.shape[1])
+
+
+# ------------------------------------------------------------------ prefix
+def prefix_sums_workspace(n: int, p: int, dtype: int, layout: int, variant: int = AUTO) -> int:
+    return int(lib().bulk_prefix_sums_workspace(n, p, dtype, layout, variant))
+
+
+def prefix_sums(x: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, out: torch.Tensor | None = None,
+                workspace: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """Inclusive prefix sums of every instance.  x is [p, n]
+    (ROW_WISE) or [n, p] (COLUMN_WISE); out may be x (in place)."""
+    _need_cuda(x)
+    n, p = _shape_np(x, layout)
+    dt = _dtype_code(x)
+    if out is None:
+        out = torch.empty_like(x)
+    _need_cuda(out)
+    need = prefix_sums_workspace(n, p, dt, layout, variant)
+    wptr, wbytes = None, 0
+    if need:
+        if workspace is None:
+            workspace = torch.empty(need, dtype=torch.uint8, device=x.device)
+        wptr, wbytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
+    _check(lib().bulk_prefix_sums(x.data_ptr(), out.data_ptr(), n, p, dt, layout, variant, wptr, wbytes,
+                                  _stream(stream)))
+    return out
+
+
+def prefix_sums_variant(n: int, p: int, dtype: int, layout: int, variant: int = AUTO) -> int:
+    return int(lib().bulk_prefix_sums_variant(n, p, dtype, layout, variant, None, None))
+
+
+def prefix_sums_host(x_host: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO,
+                     out_host: torch.Tensor | None = None, device_buf: torch.Tensor | None = None,
+                     stream=None) -> torch.Tensor:
+    """End-to-end on host (ideally pinned) buffers: H2D, kernels, D2H pipelined
+    inside the library; returns when out_host holds the result."""
+    n, p = _shape_np(x_host, layout)
+    dt = _dtype_code(x_host)
+    if out_host is None:
+        out_host = torch.empty_like(x_host)
+    if device_buf is None:
+        need = n * p * 4 + 2 * prefix_sums_workspace(n, (p + 7) // 8 + 128, dt, layout, variant)
+        device_buf = torch.empty(need, dtype=torch.uint8, device="cuda")
+    _check(lib().bulk_prefix_sums_host(x_host.data_ptr(), out_host.data_ptr(), n, p, dt, layout, variant,
+                                       device_buf.data_ptr(), device_buf.numel(), _stream(stream)))
+    return out_host
+
+
+# ---------------------------------------------------------- triangulation
+def _tri_shape(c: torch.Tensor, layout: int):
+    if c.dim() != 3:
+        raise ValueError("weights are [p, n, n] (ROW_WISE) or [n, n, p] (COLUMN_WISE)")
+    if layout == ROW_WISE:
+        p, n, n2 = c.shape
+    else:
+        n, n2, p = c.shape
+    if n != n2:
+        raise ValueError("weight matrices must be n x n")
+    return n, p
+
+
+def triangulation_workspace(n: int, p: int, dtype: int, layout: int, variant: int = AUTO) -> int:
+    return int(lib().bulk_triangulation_workspace(n, p, dtype, layout, variant))
+
+
+def triangulation_variant(n: int, p: int, dtype: int, layout: int, variant: int = AUTO) -> int:
+    return int(lib().bulk_triangulation_variant(n, p, dtype, layout, variant))
+
+
+def triangulation(c: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, out: torch.Tensor | None = None,
+                  workspace: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """out[h] = M_h[1, n-1] of Algorithm OPT for every instance."""
+    _need_cuda(c)
+    n, p = _tri_shape(c, layout)
+    dt = _dtype_code(c)
+    if out is None:
+        out = torch.empty(p, dtype=c.dtype, device=c.device)
+    need = triangulation_workspace(n, p, dt, layout, variant)
+    wptr, wbytes = None, 0
+    if need:
+        if workspace is None:
+            workspace = torch.empty(need, dtype=torch.uint8, device=c.device)
+        wptr, wbytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
+    _check(lib().bulk_triangulation(c.data_ptr(), out.data_ptr(), n, p, dt, layout, variant, wptr, wbytes,
+                                    _stream(stream)))
+    return out
+
+
+def triangulation_host(c_host: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO,
+                       out_host: torch.Tensor | None = None, device_buf: torch.Tensor | None = None,
+                       stream=None) -> torch.Tensor:
+    n, p = _tri_shape(c_host, layout)
+    dt = _dtype_code(c_host)
+    if out_host is None:
+        out_host = torch.empty(p, dtype=c_host.dtype).pin_memory()
+    if device_buf is None:
+        need = n * n * p * 4 + p * 4 + triangulation_workspace(n, p, dt, layout, variant)
+        device_buf = torch.empty(need, dtype=torch.uint8, device="cuda")
+    _check(lib().bulk_triangulation_host(c_host.data_ptr(), out_host.data_ptr(), n, p, dt, layout, variant,
+                                         device_buf.data_ptr(), device_buf.numel(), _stream(stream)))
+    return out_host
+
+
+# --------------------------------------------------------------- transpose
+def transpose(x: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """[rows, cols] -> [cols, rows] (row-wise <-> column-wise arrangement)."""
+    _need_cuda(x)
+    if x.dim() != 2 or x.element_size() != 4:
+        raise ValueError("transpose takes a 2-D tensor of 4-byte elements")
+    rows, cols = x.shape
+    if out is None:
+        out = torch.empty((cols, rows), dtype=x.dtype, device=x.device)
+    _check(lib().bulk_transpose(x.data_ptr(), out.data_ptr(), rows, cols, 4, _stream(stream)))
+    return out
+
+
+# ------------------------------------------------------ inputs / checksums
+def generate_prefix(n: int, p: int, seed: int, dtype=torch.float32, layout: int = ROW_WISE, kind: str = "uniform",
+                    h0: int = 0, device="cuda", out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    shape = (p, n) if layout == ROW_WISE else (n, p)
+    if out is None:
+        out = torch.empty(shape, dtype=dtype, device=device)
+    _check(lib().bulk_generate_prefix(out.data_ptr(), n, p, h0, seed, _dtype_code(out), layout, KINDS[kind],
+                                      _stream(stream)))
+    return out
+
+
+def generate_tri(n: int, p: int, seed: int, dtype=torch.float32, layout: int = ROW_WISE, h0: int = 0,
+                 device="cuda", out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    shape = (p, n, n) if layout == ROW_WISE else (n, n, p)
+    if out is None:
+        out = torch.empty(shape, dtype=dtype, device=device)
+    _check(lib().bulk_generate_tri(out.data_ptr(), n, p, h0, seed, _dtype_code(out), layout, _stream(stream)))
+    return out
+
+
+def checksum(values: torch.Tensor, layout: int = ROW_WISE, h0: int = 0, stream=None) -> torch.Tensor:
+    """Device uint64 (as int64 tensor) fingerprint; see bulkgen.checksum."""
+    _need_cuda(values)
+    if values.dim() == 1:
+        n, p = 1, values.shape[0]
+        layout = ROW_WISE
+    else:
+        n, p = _shape_np(values, layout)
+    acc = torch.zeros(1, dtype=torch.int64, device=values.device)
+    _check(lib().bulk_checksum(values.data_ptr(), n, p, h0, layout, acc.data_ptr(), _stream(stream)))
+    return acc
+
+
+def launch_count() -> int:
+    return int(lib().bulk_launch_count())
+
+
+def version() -> str:
+    return lib().bulk_version().decode()

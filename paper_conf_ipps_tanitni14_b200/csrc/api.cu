@@ -1,0 +1,352 @@
+// api.cu -- the C ABI of libbulkobl.so (include/bulkobl.h): argument
+// validation, variant resolution, stream-ordered launches, and the pipelined
+// host-buffer entry points.  No computation happens on the CPU.
+#include "common.cuh"
+
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+namespace bo {
+
+// ---------------------------------------------------------------- errors
+static thread_local std::string t_err;
+std::atomic<uint64_t> g_launches{0};
+
+void set_error(const std::string &msg) { t_err = msg; }
+int fail(int status, const std::string &msg) {
+    set_error(msg);
+    return status;
+}
+int cuda_check(cudaError_t e, const char *what) {
+    if (e == cudaSuccess) return BO_OK;
+    return fail(BO_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+// ---------------------------------------------------------------- TMA maps
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            p = nullptr;
+        return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    }();
+    return fn;
+}
+
+bool make_tmap_2d(CUtensorMap *map, const void *base, uint64_t rows, uint64_t cols, uint32_t box_rows,
+                  uint32_t box_cols, CUtensorMapSwizzle swz) {
+    auto fn = encode_fn();
+    if (!fn) return false;
+    cuuint64_t dims[2] = {cols, rows};
+    cuuint64_t strides[1] = {cols * 4};
+    cuuint32_t box[2] = {box_cols, box_rows};
+    cuuint32_t es[2] = {1, 1};
+    CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void *>(base), dims, strides, box, es,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+// ---------------------------------------------------------------- internals
+int launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, cudaStream_t st);
+int prefix_dispatch(const void *src, void *dst, int64_t n, int64_t p, int dtype, int layout, int variant,
+                    void *ws, cudaStream_t st);
+int resolve_prefix_variant(int64_t n, int64_t p, int layout, int variant, const void *src, const void *dst);
+int tri_dispatch(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int variant, void *ws,
+                 cudaStream_t st);
+int resolve_tri_variant(int64_t n, int64_t p, int dtype, int layout, int variant);
+size_t tri_workspace(int64_t n, int64_t p, int variant);
+int launch_gen_prefix(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
+int launch_gen_tri(void *, int64_t, int64_t, int64_t, uint64_t, int, int, cudaStream_t);
+int launch_checksum(const void *, int64_t, int64_t, int64_t, int, uint64_t *, cudaStream_t);
+
+static constexpr int64_t kMaxElems = int64_t(1) << 40;
+
+static bool valid_dtype(int d) { return d == BO_I32 || d == BO_F32; }
+static bool valid_layout(int l) { return l == BO_ROW_WISE || l == BO_COLUMN_WISE; }
+
+static bool ranges_partially_overlap(const void *a, const void *b, size_t bytes) {
+    const uintptr_t x = reinterpret_cast<uintptr_t>(a), y = reinterpret_cast<uintptr_t>(b);
+    if (x == y) return false;
+    return x < y + bytes && y < x + bytes;
+}
+
+static int check_prefix_args(const void *src, const void *dst, int64_t n, int64_t p, int dtype, int layout,
+                             int variant) {
+    if (n < 0 || p < 0) return fail(BO_EINVAL, "prefix: n and p must be >= 0");
+    if (!valid_dtype(dtype)) return fail(BO_EINVAL, "prefix: dtype must be BO_I32 or BO_F32");
+    if (!valid_layout(layout)) return fail(BO_EINVAL, "prefix: layout must be BO_ROW_WISE or BO_COLUMN_WISE");
+    if (n > 0 && p > kMaxElems / n) return fail(BO_EINVAL, "prefix: n*p too large");
+    if (n * p > 0 && (!src || !dst)) return fail(BO_EINVAL, "prefix: NULL pointer");
+    if (n * p > 0 && ranges_partially_overlap(src, dst, static_cast<size_t>(n * p) * 4))
+        return fail(BO_EINVAL, "prefix: src and dst partially overlap");
+    switch (variant) {
+        case BO_AUTO:
+        case BO_PS_NAIVE:
+            return BO_OK;
+        case BO_PS_ACROSS:
+            if (layout != BO_COLUMN_WISE) return fail(BO_EUNSUPPORTED, "prefix ACROSS needs the column-wise layout");
+            return BO_OK;
+        case BO_PS_WARPSCAN:
+        case BO_PS_FUSED_ROW:
+        case BO_PS_TRANSPOSED:
+            if (layout != BO_ROW_WISE) return fail(BO_EUNSUPPORTED, "prefix variant needs the row-wise layout");
+            return BO_OK;
+        default:
+            return fail(BO_EINVAL, "prefix: unknown variant");
+    }
+}
+
+static int check_tri_args(const void *c, const void *out, int64_t n, int64_t p, int dtype, int layout,
+                          int variant) {
+    if (n < 3 || n > 4096) return fail(BO_EINVAL, "triangulation: need 3 <= n <= 4096");
+    if (p < 0) return fail(BO_EINVAL, "triangulation: p must be >= 0");
+    if (!valid_dtype(dtype)) return fail(BO_EINVAL, "triangulation: dtype must be BO_I32 or BO_F32");
+    if (!valid_layout(layout)) return fail(BO_EINVAL, "triangulation: bad layout");
+    if (p > kMaxElems / (n * n)) return fail(BO_EINVAL, "triangulation: n*n*p too large");
+    if (p > 0 && (!c || !out)) return fail(BO_EINVAL, "triangulation: NULL pointer");
+    if (variant != BO_AUTO && (variant < BO_TRI_UMM_GLOBAL || variant > BO_TRI_TILED))
+        return fail(BO_EINVAL, "triangulation: unknown variant");
+    return BO_OK;
+}
+
+static size_t prefix_ws(int64_t n, int64_t p, int variant) {
+    return variant == BO_PS_TRANSPOSED ? static_cast<size_t>(n) * p * 4 : 0;
+}
+
+// Internal streams for the host-buffer pipeline (one pair per device).
+struct HostPipe {
+    cudaStream_t s[2] = {nullptr, nullptr};
+    cudaEvent_t ev_start = nullptr, ev_done[2] = {nullptr, nullptr};
+};
+static HostPipe *host_pipe() {
+    static std::mutex mu;
+    static std::vector<HostPipe *> pipes;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> g(mu);
+    if (static_cast<int>(pipes.size()) <= dev) pipes.resize(dev + 1, nullptr);
+    if (!pipes[dev]) {
+        auto *hp = new HostPipe;
+        for (int i = 0; i < 2; ++i) {
+            cudaStreamCreateWithFlags(&hp->s[i], cudaStreamNonBlocking);
+            cudaEventCreateWithFlags(&hp->ev_done[i], cudaEventDisableTiming);
+        }
+        cudaEventCreateWithFlags(&hp->ev_start, cudaEventDisableTiming);
+        pipes[dev] = hp;
+    }
+    return pipes[dev];
+}
+
+static int64_t host_chunk(int64_t p) {
+    // ~8 chunks, multiple of 128 instances, so copies of chunk k+1 overlap compute/copy-back of chunk k
+    int64_t ch = (p + 7) / 8;
+    ch = ((ch + 127) / 128) * 128;
+    return std::max<int64_t>(std::min<int64_t>(ch, p), 1);
+}
+
+}  // namespace bo
+
+using namespace bo;
+
+extern "C" {
+
+const char *bulk_last_error(void) { return t_err.c_str(); }
+uint64_t bulk_launch_count(void) { return g_launches.load(); }
+const char *bulk_version(void) { return "bulkobl 0.1 (sm_100a)"; }
+
+int bulk_prefix_sums_variant(int64_t n, int64_t p, int dtype, int layout, int variant, const void *src,
+                             const void *dst) {
+    (void)dtype;
+    return resolve_prefix_variant(n, p, layout, variant, src, dst);
+}
+
+size_t bulk_prefix_sums_workspace(int64_t n, int64_t p, int dtype, int layout, int variant) {
+    (void)dtype;
+    return prefix_ws(n, p, resolve_prefix_variant(n, p, layout, variant, nullptr, nullptr));
+}
+
+int bulk_prefix_sums(const void *src, void *dst, int64_t n, int64_t p, int dtype, int layout, int variant,
+                     void *workspace, size_t workspace_bytes, void *stream) {
+    t_err.clear();
+    int rc = check_prefix_args(src, dst, n, p, dtype, layout, variant);
+    if (rc) return rc;
+    if (n * p == 0) return BO_OK;
+    const int v = resolve_prefix_variant(n, p, layout, variant, src, dst);
+    const size_t need = prefix_ws(n, p, v);
+    if (need > 0 && (!workspace || workspace_bytes < need))
+        return fail(BO_EINVAL, "prefix: workspace too small (need " + std::to_string(need) + " bytes)");
+    if (need > 0 && (ranges_partially_overlap(workspace, src, need) || workspace == src || workspace == dst))
+        return fail(BO_EINVAL, "prefix: workspace overlaps the data");
+    return prefix_dispatch(src, dst, n, p, dtype, layout, v, workspace, static_cast<cudaStream_t>(stream));
+}
+
+int bulk_triangulation_variant(int64_t n, int64_t p, int dtype, int layout, int variant) {
+    return resolve_tri_variant(n, p, dtype, layout, variant);
+}
+
+size_t bulk_triangulation_workspace(int64_t n, int64_t p, int dtype, int layout, int variant) {
+    if (n < 3 || p < 0) return 0;
+    return tri_workspace(n, p, resolve_tri_variant(n, p, dtype, layout, variant));
+}
+
+int bulk_triangulation(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int variant,
+                       void *workspace, size_t workspace_bytes, void *stream) {
+    t_err.clear();
+    int rc = check_tri_args(c, out, n, p, dtype, layout, variant);
+    if (rc) return rc;
+    if (p == 0) return BO_OK;
+    const int v = resolve_tri_variant(n, p, dtype, layout, variant);
+    const size_t need = tri_workspace(n, p, v);
+    if (need > 0 && (!workspace || workspace_bytes < need))
+        return fail(BO_EINVAL, "triangulation: workspace too small (need " + std::to_string(need) + " bytes)");
+    return tri_dispatch(c, out, n, p, dtype, layout, v, workspace, static_cast<cudaStream_t>(stream));
+}
+
+int bulk_transpose(const void *src, void *dst, int64_t rows, int64_t cols, size_t elem_bytes, void *stream) {
+    t_err.clear();
+    if (elem_bytes != 4) return fail(BO_EUNSUPPORTED, "transpose: only 4-byte elements");
+    if (rows < 0 || cols < 0) return fail(BO_EINVAL, "transpose: rows and cols must be >= 0");
+    if (rows > 0 && cols > kMaxElems / rows) return fail(BO_EINVAL, "transpose: rows*cols too large");
+    if (rows * cols == 0) return BO_OK;
+    if (!src || !dst) return fail(BO_EINVAL, "transpose: NULL pointer");
+    if (src == dst || ranges_partially_overlap(src, dst, static_cast<size_t>(rows * cols) * 4))
+        return fail(BO_EINVAL, "transpose: src and dst overlap (out of place only)");
+    return launch_transpose(src, dst, rows, cols, static_cast<cudaStream_t>(stream));
+}
+
+int bulk_generate_prefix(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout,
+                         int kind, void *stream) {
+    t_err.clear();
+    if (n < 0 || p < 0 || h0 < 0 || !valid_dtype(dtype) || !valid_layout(layout) || kind < 0 || kind > 3)
+        return fail(BO_EINVAL, "generate_prefix: bad argument");
+    if (n * p > 0 && !dst) return fail(BO_EINVAL, "generate_prefix: NULL pointer");
+    return launch_gen_prefix(dst, n, p, h0, seed, dtype, layout, kind, static_cast<cudaStream_t>(stream));
+}
+
+int bulk_generate_tri(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout,
+                      void *stream) {
+    t_err.clear();
+    if (n < 1 || p < 0 || h0 < 0 || !valid_dtype(dtype) || !valid_layout(layout))
+        return fail(BO_EINVAL, "generate_tri: bad argument");
+    if (p > 0 && !dst) return fail(BO_EINVAL, "generate_tri: NULL pointer");
+    return launch_gen_tri(dst, n, p, h0, seed, dtype, layout, static_cast<cudaStream_t>(stream));
+}
+
+int bulk_checksum(const void *values, int64_t n, int64_t p, int64_t h0, int layout, uint64_t *acc, void *stream) {
+    t_err.clear();
+    if (n < 0 || p < 0 || h0 < 0 || !valid_layout(layout) || !acc) return fail(BO_EINVAL, "checksum: bad argument");
+    if (n * p > 0 && !values) return fail(BO_EINVAL, "checksum: NULL pointer");
+    return launch_checksum(values, n, p, h0, layout, acc, static_cast<cudaStream_t>(stream));
+}
+
+// ------------------------------------------------------------------ host e2e
+int bulk_prefix_sums_host(const void *h_src, void *h_dst, int64_t n, int64_t p, int dtype, int layout,
+                          int variant, void *d_buf, size_t d_bytes, void *stream) {
+    t_err.clear();
+    int rc = check_prefix_args(h_src, h_dst, n, p, dtype, layout, variant);
+    if (rc) return rc;
+    if (n * p == 0) return BO_OK;
+    const int v = resolve_prefix_variant(n, p, layout, variant, nullptr, nullptr);
+    const int64_t ch = host_chunk(p);
+    const size_t data_bytes = static_cast<size_t>(n) * p * 4;
+    const size_t ws_chunk = prefix_ws(n, ch, v);
+    if (!d_buf || d_bytes < data_bytes + 2 * ws_chunk)
+        return fail(BO_EINVAL, "prefix_host: device buffer too small (need " +
+                                   std::to_string(data_bytes + 2 * ws_chunk) + " bytes)");
+    HostPipe *hp = host_pipe();
+    cudaStream_t caller = static_cast<cudaStream_t>(stream);
+    if ((rc = cuda_check(cudaEventRecord(hp->ev_start, caller), "prefix_host: event"))) return rc;
+    for (int i = 0; i < 2; ++i)
+        if ((rc = cuda_check(cudaStreamWaitEvent(hp->s[i], hp->ev_start, 0), "prefix_host: wait"))) return rc;
+    const char *hs = static_cast<const char *>(h_src);
+    char *hd = static_cast<char *>(h_dst);
+    char *db = static_cast<char *>(d_buf);
+    int k = 0;
+    for (int64_t p0 = 0; p0 < p; p0 += ch, ++k) {
+        const int64_t pc = std::min(ch, p - p0);
+        cudaStream_t s = hp->s[k & 1];
+        char *dchunk = db + static_cast<size_t>(p0) * n * 4;        // compact chunk, same layout
+        void *ws = ws_chunk ? db + data_bytes + (k & 1) * ws_chunk : nullptr;
+        if (layout == BO_ROW_WISE) {
+            rc = cuda_check(cudaMemcpyAsync(dchunk, hs + static_cast<size_t>(p0) * n * 4,
+                                            static_cast<size_t>(pc) * n * 4, cudaMemcpyHostToDevice, s),
+                            "prefix_host: H2D");
+        } else {
+            rc = cuda_check(cudaMemcpy2DAsync(dchunk, pc * 4, hs + p0 * 4, p * 4, pc * 4, n, cudaMemcpyHostToDevice, s),
+                            "prefix_host: H2D");
+        }
+        if (rc) return rc;
+        if ((rc = prefix_dispatch(dchunk, dchunk, n, pc, dtype, layout, v, ws, s))) return rc;
+        if (layout == BO_ROW_WISE) {
+            rc = cuda_check(cudaMemcpyAsync(hd + static_cast<size_t>(p0) * n * 4, dchunk,
+                                            static_cast<size_t>(pc) * n * 4, cudaMemcpyDeviceToHost, s),
+                            "prefix_host: D2H");
+        } else {
+            rc = cuda_check(cudaMemcpy2DAsync(hd + p0 * 4, p * 4, dchunk, pc * 4, pc * 4, n, cudaMemcpyDeviceToHost, s),
+                            "prefix_host: D2H");
+        }
+        if (rc) return rc;
+    }
+    for (int i = 0; i < 2; ++i) {
+        if ((rc = cuda_check(cudaEventRecord(hp->ev_done[i], hp->s[i]), "prefix_host: event"))) return rc;
+        if ((rc = cuda_check(cudaStreamWaitEvent(caller, hp->ev_done[i], 0), "prefix_host: wait"))) return rc;
+    }
+    return cuda_check(cudaStreamSynchronize(caller), "prefix_host: sync");
+}
+
+int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, int dtype, int layout,
+                            int variant, void *d_buf, size_t d_bytes, void *stream) {
+    t_err.clear();
+    int rc = check_tri_args(h_c, h_out, n, p, dtype, layout, variant);
+    if (rc) return rc;
+    if (p == 0) return BO_OK;
+    const int v = resolve_tri_variant(n, p, dtype, layout, variant);
+    const int64_t ch = host_chunk(p);
+    const size_t nn = static_cast<size_t>(n) * n;
+    const size_t c_bytes = nn * p * 4, out_bytes = static_cast<size_t>(p) * 4;
+    const size_t ws_bytes = tri_workspace(n, p, v);
+    if (!d_buf || d_bytes < c_bytes + out_bytes + ws_bytes)
+        return fail(BO_EINVAL, "triangulation_host: device buffer too small (need " +
+                                   std::to_string(c_bytes + out_bytes + ws_bytes) + " bytes)");
+    HostPipe *hp = host_pipe();
+    cudaStream_t caller = static_cast<cudaStream_t>(stream);
+    if ((rc = cuda_check(cudaEventRecord(hp->ev_start, caller), "tri_host: event"))) return rc;
+    for (int i = 0; i < 2; ++i)
+        if ((rc = cuda_check(cudaStreamWaitEvent(hp->s[i], hp->ev_start, 0), "tri_host: wait"))) return rc;
+    const char *hc = static_cast<const char *>(h_c);
+    char *ho = static_cast<char *>(h_out);
+    char *db = static_cast<char *>(d_buf);
+    char *dout = db + c_bytes;
+    char *dws = db + c_bytes + out_bytes;
+    int k = 0;
+    for (int64_t p0 = 0; p0 < p; p0 += ch, ++k) {
+        const int64_t pc = std::min(ch, p - p0);
+        cudaStream_t s = hp->s[k & 1];
+        char *dchunk = db + static_cast<size_t>(p0) * nn * 4;
+        if (layout == BO_ROW_WISE)
+            rc = cuda_check(cudaMemcpyAsync(dchunk, hc + static_cast<size_t>(p0) * nn * 4, pc * nn * 4,
+                                            cudaMemcpyHostToDevice, s),
+                            "tri_host: H2D");
+        else
+            rc = cuda_check(cudaMemcpy2DAsync(dchunk, pc * 4, hc + p0 * 4, p * 4, pc * 4, nn, cudaMemcpyHostToDevice, s),
+                            "tri_host: H2D");
+        if (rc) return rc;
+        void *ws = ws_bytes ? dws + static_cast<size_t>(p0) * (n - 1) * (n - 1) * 4 : nullptr;
+        if ((rc = tri_dispatch(dchunk, dout + p0 * 4, n, pc, dtype, layout, v, ws, s))) return rc;
+        if ((rc = cuda_check(cudaMemcpyAsync(ho + p0 * 4, dout + p0 * 4, pc * 4, cudaMemcpyDeviceToHost, s),
+                             "tri_host: D2H")))
+            return rc;
+    }
+    for (int i = 0; i < 2; ++i) {
+        if ((rc = cuda_check(cudaEventRecord(hp->ev_done[i], hp->s[i]), "tri_host: event"))) return rc;
+        if ((rc = cuda_check(cudaStreamWaitEvent(caller, hp->ev_done[i], 0), "tri_host: wait"))) return rc;
+    }
+    return cuda_check(cudaStreamSynchronize(caller), "tri_host: sync");
+}
+
+}  // extern "C"

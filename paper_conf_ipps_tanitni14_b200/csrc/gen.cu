@@ -1,0 +1,115 @@
+// gen.cu -- device side of the counter-based input generator (bulkgen/) and
+// the order-independent result checksum.  Neither holds any of
+// the method's arithmetic; both exist so that inputs never cross PCIe/NVLink
+// and every rank can fingerprint its shard.
+#include "common.cuh"
+
+namespace bo {
+
+constexpr uint64_t kSeedMul = 0x9E3779B97F4A7C15ull;
+constexpr uint64_t kHMul = 0xD1B54A32D192ED03ull;
+constexpr uint64_t kEMul = 0x8CB92BA72F3D8DD7ull;
+
+__device__ __forceinline__ uint64_t mix64(uint64_t z) {
+    z ^= z >> 30;
+    z *= 0xBF58476D1CE4E5B9ull;
+    z ^= z >> 27;
+    z *= 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    return z;
+}
+
+__device__ __forceinline__ uint64_t gen_u(uint64_t seed, uint64_t h, uint64_t e) {
+    return mix64(seed * kSeedMul + h * kHMul + e * kEMul);
+}
+
+__global__ void gen_prefix_kernel(uint32_t *dst, long long n, long long p, long long h0, uint64_t seed,
+                                  int dtype, int layout, int kind) {
+    const long long total = n * p;
+    for (long long idx = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; idx < total;
+         idx += static_cast<long long>(gridDim.x) * blockDim.x) {
+        long long h, e;
+        if (layout == BO_ROW_WISE) { h = idx / n; e = idx - h * n; }
+        else { e = idx / p; h = idx - e * p; }
+        const uint64_t u = gen_u(seed, static_cast<uint64_t>(h0 + h), static_cast<uint64_t>(e));
+        uint32_t bits;
+        if (kind == 0) {
+            bits = dtype == BO_I32 ? static_cast<uint32_t>(u >> 32)
+                                   : __float_as_uint(static_cast<float>(u >> 40) * 0x1p-24f);
+        } else if (kind == 1) {
+            bits = dtype == BO_I32 ? 1u : __float_as_uint(1.0f);
+        } else if (kind == 2) {
+            bits = dtype == BO_I32 ? static_cast<uint32_t>(e) : __float_as_uint(static_cast<float>(e));
+        } else {
+            const uint32_t v = static_cast<uint32_t>(u >> 60);
+            bits = dtype == BO_I32 ? v : __float_as_uint(static_cast<float>(v));
+        }
+        dst[idx] = bits;
+    }
+}
+
+__global__ void gen_tri_kernel(uint32_t *dst, long long n, long long p, long long h0, uint64_t seed, int dtype,
+                               int layout) {
+    const long long nn = n * n, total = nn * p;
+    for (long long idx = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; idx < total;
+         idx += static_cast<long long>(gridDim.x) * blockDim.x) {
+        long long h, e;
+        if (layout == BO_ROW_WISE) { h = idx / nn; e = idx - h * nn; }
+        else { e = idx / p; h = idx - e * p; }
+        const long long a = e / n, b = e - a * n;
+        uint32_t bits = 0;
+        if (b - a >= 2 && !(a == 0 && b == n - 1)) {
+            const uint64_t u = gen_u(seed, static_cast<uint64_t>(h0 + h), static_cast<uint64_t>(e));
+            bits = dtype == BO_I32 ? static_cast<uint32_t>(u >> 44)
+                                   : __float_as_uint(static_cast<float>(u >> 40) * 0x1p-24f);
+        }
+        dst[idx] = bits;
+    }
+}
+
+__global__ void checksum_kernel(const uint32_t *v, long long n, long long p, long long h0, int layout,
+                                unsigned long long *acc) {
+    const long long total = n * p;
+    uint64_t local = 0;
+    for (long long idx = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; idx < total;
+         idx += static_cast<long long>(gridDim.x) * blockDim.x) {
+        long long h, e;
+        if (layout == BO_ROW_WISE) { h = idx / n; e = idx - h * n; }
+        else { e = idx / p; h = idx - e * p; }
+        local += mix64(static_cast<uint64_t>(v[idx]) * kSeedMul + static_cast<uint64_t>(h0 + h) * kHMul +
+                       static_cast<uint64_t>(e) * kEMul);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) local += __shfl_xor_sync(0xffffffffu, local, o);
+    if ((threadIdx.x & 31) == 0) atomicAdd(acc, static_cast<unsigned long long>(local));
+}
+
+static unsigned grid_for(long long total) {
+    const long long g = (total + 255) / 256;
+    return static_cast<unsigned>(std::max<long long>(1, std::min<long long>(g, 64LL * num_sms())));
+}
+
+int launch_gen_prefix(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout, int kind,
+                      cudaStream_t st) {
+    if (n * p == 0) return BO_OK;
+    gen_prefix_kernel<<<grid_for(n * p), 256, 0, st>>>(static_cast<uint32_t *>(dst), n, p, h0, seed, dtype, layout,
+                                                       kind);
+    return after_launch("gen_prefix_kernel");
+}
+
+int launch_gen_tri(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout,
+                   cudaStream_t st) {
+    if (n * n * p == 0) return BO_OK;
+    gen_tri_kernel<<<grid_for(n * n * p), 256, 0, st>>>(static_cast<uint32_t *>(dst), n, p, h0, seed, dtype,
+                                                        layout);
+    return after_launch("gen_tri_kernel");
+}
+
+int launch_checksum(const void *v, int64_t n, int64_t p, int64_t h0, int layout, uint64_t *acc, cudaStream_t st) {
+    if (n * p == 0) return BO_OK;
+    checksum_kernel<<<grid_for(n * p), 256, 0, st>>>(static_cast<const uint32_t *>(v), n, p, h0, layout,
+                                                     reinterpret_cast<unsigned long long *>(acc));
+    return after_launch("checksum_kernel");
+}
+
+}  // namespace bo

@@ -1,0 +1,360 @@
+// prefix.cu -- bulk inclusive prefix sums (Algorithm Prefix-sums, P:95-102;
+// Parallel Algorithm Prefix-sums).
+//
+// Every variant except WARPSCAN keeps the paper's left-to-right order
+// r <- r + b[i] per instance, so fp32 results are bit-identical to the
+// sequential algorithm.  int32 adds wrap mod 2^32.
+//
+//  ACROSS     column-wise [n][p]: thread owns 4 adjacent instances,
+//             one 128-bit coalesced load/store per row i, U rows of loads in
+//             flight (the addresses are input-independent -- obliviousness,
+//             so they can be issued far ahead of the adds).
+//  FUSED_ROW  row-wise [p][n]: TMA brings [128 instances x 32 elems]
+//             boxes (128B swizzle) into a smem ring; thread t scans instance t
+//             sequentially out of smem (conflict-free 128-bit reads), writes
+//             in place, TMA stores the box.  The row->column transpose happens
+//             on chip: HBM traffic = 2*n*p*4 bytes, same as column-wise.
+//  WARPSCAN   row-wise: warp per instance, shuffle scan (fp32 reassociated).
+//  NAIVE      the paper's kernel: one thread per instance, scalar accesses in
+//             the given arrangement -- the prior-art baseline.
+#include "common.cuh"
+
+namespace bo {
+
+int launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, cudaStream_t st);
+
+template <typename T>
+__device__ __forceinline__ T bits_as(uint32_t u) {
+    if constexpr (sizeof(T) == 4 && std::is_same<T, float>::value) return __uint_as_float(u);
+    else return static_cast<T>(u);
+}
+template <typename T>
+__device__ __forceinline__ uint32_t as_bits(T v) {
+    if constexpr (std::is_same<T, float>::value) return __float_as_uint(v);
+    else return static_cast<uint32_t>(v);
+}
+
+// ------------------------------------------------------------------ ACROSS
+template <typename T, int U>
+__global__ void __launch_bounds__(256)
+ps_across_vec4(const T *src, T *dst, long long n, long long p4) {
+    const long long g = blockIdx.x * 256LL + threadIdx.x;
+    if (g >= p4) return;
+    const uint4 *s = reinterpret_cast<const uint4 *>(src) + g;
+    uint4 *d = reinterpret_cast<uint4 *>(dst) + g;
+    T r0 = T(0), r1 = T(0), r2 = T(0), r3 = T(0);
+    long long i = 0;
+    for (; i + U <= n; i += U) {
+        uint4 v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[u] = __ldcs(s + (i + u) * p4);
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            r0 = add_wrap(r0, bits_as<T>(v[u].x));
+            r1 = add_wrap(r1, bits_as<T>(v[u].y));
+            r2 = add_wrap(r2, bits_as<T>(v[u].z));
+            r3 = add_wrap(r3, bits_as<T>(v[u].w));
+            __stcs(d + (i + u) * p4, make_uint4(as_bits(r0), as_bits(r1), as_bits(r2), as_bits(r3)));
+        }
+    }
+    for (; i < n; ++i) {
+        const uint4 v = __ldcs(s + i * p4);
+        r0 = add_wrap(r0, bits_as<T>(v.x));
+        r1 = add_wrap(r1, bits_as<T>(v.y));
+        r2 = add_wrap(r2, bits_as<T>(v.z));
+        r3 = add_wrap(r3, bits_as<T>(v.w));
+        __stcs(d + i * p4, make_uint4(as_bits(r0), as_bits(r1), as_bits(r2), as_bits(r3)));
+    }
+}
+
+template <typename T, int U>
+__global__ void __launch_bounds__(256)
+ps_across_scalar(const T *src, T *dst, long long n, long long p) {
+    const long long j = blockIdx.x * 256LL + threadIdx.x;
+    if (j >= p) return;
+    T r = T(0);
+    long long i = 0;
+    for (; i + U <= n; i += U) {
+        T v[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[u] = src[(i + u) * p + j];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            r = add_wrap(r, v[u]);
+            dst[(i + u) * p + j] = r;
+        }
+    }
+    for (; i < n; ++i) {
+        r = add_wrap(r, src[i * p + j]);
+        dst[i * p + j] = r;
+    }
+}
+
+// --------------------------------------------------------------- FUSED_ROW
+namespace fr {
+constexpr int kInst = 128;                 // instances per tile = threads per CTA
+constexpr int kElems = 32;                 // elements per chunk (128 B rows, swizzle 128B)
+constexpr int kStages = 6;
+constexpr uint32_t kBoxBytes = kInst * kElems * 4;   // 16 KiB
+constexpr size_t kSmem = 1024 + kStages * kBoxBytes + kStages * 8;
+}  // namespace fr
+
+template <typename T>
+__global__ void __launch_bounds__(fr::kInst)
+ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant__ CUtensorMap dst_map,
+                 long long ntiles, int nchunks) {
+    using namespace fr;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                               ~uintptr_t(1023));
+    uint64_t *full = reinterpret_cast<uint64_t *>(buf + kStages * kBoxBytes);
+    const int tid = threadIdx.x;
+    const long long first = blockIdx.x;
+    const long long my_tiles = ntiles > first ? (ntiles - 1 - first) / gridDim.x + 1 : 0;
+    const long long items = my_tiles * nchunks;
+
+    if (tid == 0) {
+        prefetch_tmap(&src_map);
+        prefetch_tmap(&dst_map);
+        for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
+        fence_barrier_init();
+    }
+    __syncthreads();
+
+    auto coords = [&](long long i, int &c0, int &c1) {
+        const long long tile = first + (i / nchunks) * gridDim.x;
+        c0 = static_cast<int>(i % nchunks) * kElems;
+        c1 = static_cast<int>(tile * kInst);
+    };
+    auto issue_load = [&](long long i) {
+        int c0, c1;
+        coords(i, c0, c1);
+        const int s = static_cast<int>(i % kStages);
+        mbar_arrive_expect_tx(&full[s], kBoxBytes);
+        tma_load_2d(buf + s * kBoxBytes, &src_map, c0, c1, &full[s]);
+    };
+    if (tid == 0)
+        for (long long i = 0; i < items && i < kStages - 1; ++i) issue_load(i);
+
+    T r = T(0);
+    for (long long i = 0; i < items; ++i) {
+        const int s = static_cast<int>(i % kStages);
+        if (i % nchunks == 0) r = T(0);                 // new tile: r_j <- 0
+        mbar_wait(&full[s], static_cast<uint32_t>((i / kStages) & 1));
+        uint8_t *box = buf + s * kBoxBytes;
+#pragma unroll
+        for (int k = 0; k < kElems / 4; ++k) {
+            uint4 *q = reinterpret_cast<uint4 *>(box + swz128(tid, k));
+            uint4 v = *q;
+            r = add_wrap(r, bits_as<T>(v.x)); v.x = as_bits(r);   // r <- r + b[i]; b[i] <- r
+            r = add_wrap(r, bits_as<T>(v.y)); v.y = as_bits(r);
+            r = add_wrap(r, bits_as<T>(v.z)); v.z = as_bits(r);
+            r = add_wrap(r, bits_as<T>(v.w)); v.w = as_bits(r);
+            *q = v;
+        }
+        fence_proxy_async_smem();
+        __syncthreads();
+        if (tid == 0) {
+            int c0, c1;
+            coords(i, c0, c1);
+            tma_store_2d(&dst_map, box, c0, c1);
+            bulk_commit();
+            bulk_wait_read<1>();                       // store i-1 no longer reads its stage
+            if (i + kStages - 1 < items) issue_load(i + kStages - 1);
+        }
+    }
+    if (tid == 0) bulk_wait<0>();
+}
+
+// Fallback for any n / alignment: coalesced warp loads into a padded tile.
+template <typename T>
+__global__ void __launch_bounds__(128)
+ps_fused_row_smem(const T *src, T *dst, long long n, long long p) {
+    __shared__ T tile[128][33];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    for (long long t0 = blockIdx.x * 128LL; t0 < p; t0 += 128LL * gridDim.x) {
+        T r = T(0);
+        for (long long c0 = 0; c0 < n; c0 += 32) {
+            for (int row = warp; row < 128; row += 4) {
+                const long long h = t0 + row, c = c0 + lane;
+                tile[row][lane] = (h < p && c < n) ? src[h * n + c] : T(0);
+            }
+            __syncthreads();
+#pragma unroll 8
+            for (int e = 0; e < 32; ++e) {
+                r = add_wrap(r, tile[tid][e]);
+                tile[tid][e] = r;
+            }
+            __syncthreads();
+            for (int row = warp; row < 128; row += 4) {
+                const long long h = t0 + row, c = c0 + lane;
+                if (h < p && c < n) dst[h * n + c] = tile[row][lane];
+            }
+            __syncthreads();
+        }
+    }
+}
+
+// ---------------------------------------------------------------- WARPSCAN
+template <typename T>
+__device__ __forceinline__ T warp_incl_scan(T x, int lane) {
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const T y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x = add_wrap(y, x);
+    }
+    return x;
+}
+
+template <typename T, bool kVec>
+__global__ void __launch_bounds__(256)
+ps_warpscan(const T *src, T *dst, long long n, long long p) {
+    const int lane = threadIdx.x & 31;
+    const long long warps = (static_cast<long long>(gridDim.x) * blockDim.x) >> 5;
+    for (long long h = (blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x) >> 5; h < p;
+         h += warps) {
+        const T *s = src + h * n;
+        T *d = dst + h * n;
+        T carry = T(0);
+        if (kVec) {
+            for (long long c = 0; c < n; c += 128) {
+                const long long idx = c + lane * 4;
+                uint4 v = idx < n ? __ldcs(reinterpret_cast<const uint4 *>(s + idx)) : make_uint4(0, 0, 0, 0);
+                T a = bits_as<T>(v.x), b = bits_as<T>(v.y), e = bits_as<T>(v.z), f = bits_as<T>(v.w);
+                b = add_wrap(a, b);
+                e = add_wrap(b, e);
+                f = add_wrap(e, f);
+                const T incl = warp_incl_scan(f, lane);
+                T excl = __shfl_up_sync(0xffffffffu, incl, 1);
+                excl = lane == 0 ? carry : add_wrap(carry, excl);
+                if (idx < n)
+                    __stcs(reinterpret_cast<uint4 *>(d + idx),
+                           make_uint4(as_bits(add_wrap(excl, a)), as_bits(add_wrap(excl, b)),
+                                      as_bits(add_wrap(excl, e)), as_bits(add_wrap(excl, f))));
+                carry = add_wrap(carry, __shfl_sync(0xffffffffu, incl, 31));
+            }
+        } else {
+            for (long long c = 0; c < n; c += 32) {
+                const long long idx = c + lane;
+                const T v = idx < n ? s[idx] : T(0);
+                const T incl = warp_incl_scan(v, lane);
+                if (idx < n) d[idx] = add_wrap(carry, incl);
+                carry = add_wrap(carry, __shfl_sync(0xffffffffu, incl, 31));
+            }
+        }
+    }
+}
+
+// ------------------------------------------------------------------- NAIVE
+// Parallel Algorithm Prefix-sums exactly as printed: thread T(j)
+// keeps r_j and walks its array with one 32-bit access per step.
+template <typename T>
+__global__ void __launch_bounds__(64)
+ps_naive(const T *src, T *dst, long long n, long long p, int layout) {
+    const long long j = blockIdx.x * 64LL + threadIdx.x;
+    if (j >= p) return;
+    T r = T(0);
+    for (long long i = 0; i < n; ++i) {
+        const long long a = layout == BO_ROW_WISE ? j * n + i : i * p + j;
+        r = add_wrap(r, src[a]);
+        dst[a] = r;
+    }
+}
+
+// ------------------------------------------------------------------- host
+bool fused_tma_ok(const void *src, const void *dst, int64_t n, int64_t p) {
+    return aligned16(src) && aligned16(dst) && n % 4 == 0 && n < (int64_t(1) << 31) &&
+           p < (int64_t(1) << 31);
+}
+
+int resolve_prefix_variant(int64_t n, int64_t p, int layout, int variant, const void *src, const void *dst) {
+    (void)n; (void)p; (void)src; (void)dst;
+    if (variant != BO_AUTO) return variant;
+    return layout == BO_COLUMN_WISE ? BO_PS_ACROSS : BO_PS_FUSED_ROW;
+}
+
+template <typename T>
+static int launch_across(const T *src, T *dst, int64_t n, int64_t p, cudaStream_t st) {
+    if (p % 4 == 0 && aligned16(src) && aligned16(dst)) {
+        const long long p4 = p / 4;
+        const unsigned grid = static_cast<unsigned>((p4 + 255) / 256);
+        ps_across_vec4<T, 8><<<grid, 256, 0, st>>>(src, dst, n, p4);
+        return after_launch("ps_across_vec4");
+    }
+    const unsigned grid = static_cast<unsigned>((p + 255) / 256);
+    ps_across_scalar<T, 8><<<grid, 256, 0, st>>>(src, dst, n, p);
+    return after_launch("ps_across_scalar");
+}
+
+template <typename T>
+static int launch_fused_row(const T *src, T *dst, int64_t n, int64_t p, cudaStream_t st) {
+    if (fused_tma_ok(src, dst, n, p)) {
+        CUtensorMap smap, dmap;
+        if (!make_tmap_2d(&smap, src, p, n, fr::kInst, fr::kElems, CU_TENSOR_MAP_SWIZZLE_128B) ||
+            !make_tmap_2d(&dmap, dst, p, n, fr::kInst, fr::kElems, CU_TENSOR_MAP_SWIZZLE_128B))
+            return fail(BO_ECUDA, "prefix fused-row: cuTensorMapEncodeTiled failed");
+        static bool attr = [] {
+            return cudaFuncSetAttribute(ps_fused_row_tma<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        static_cast<int>(fr::kSmem)) == cudaSuccess;
+        }();
+        if (!attr) return fail(BO_ECUDA, "prefix fused-row: cannot set dynamic smem");
+        const long long ntiles = (p + fr::kInst - 1) / fr::kInst;
+        const int nchunks = static_cast<int>((n + fr::kElems - 1) / fr::kElems);
+        const long long grid = std::min<long long>(ntiles, 2LL * num_sms());
+        ps_fused_row_tma<T><<<static_cast<unsigned>(grid), fr::kInst, fr::kSmem, st>>>(smap, dmap, ntiles,
+                                                                                     nchunks);
+        return after_launch("ps_fused_row_tma");
+    }
+    const long long blocks = std::min<long long>((p + 127) / 128, 16LL * num_sms());
+    ps_fused_row_smem<T><<<static_cast<unsigned>(blocks), 128, 0, st>>>(src, dst, n, p);
+    return after_launch("ps_fused_row_smem");
+}
+
+template <typename T>
+static int launch_warpscan(const T *src, T *dst, int64_t n, int64_t p, cudaStream_t st) {
+    const long long blocks = std::min<long long>((p + 7) / 8, 32LL * num_sms());
+    if (n % 4 == 0 && aligned16(src) && aligned16(dst))
+        ps_warpscan<T, true><<<static_cast<unsigned>(blocks), 256, 0, st>>>(src, dst, n, p);
+    else
+        ps_warpscan<T, false><<<static_cast<unsigned>(blocks), 256, 0, st>>>(src, dst, n, p);
+    return after_launch("ps_warpscan");
+}
+
+template <typename T>
+static int run_prefix(const T *src, T *dst, int64_t n, int64_t p, int layout, int variant, void *ws,
+                      cudaStream_t st) {
+    switch (variant) {
+        case BO_PS_ACROSS:
+            return launch_across(src, dst, n, p, st);
+        case BO_PS_FUSED_ROW:
+            return launch_fused_row(src, dst, n, p, st);
+        case BO_PS_WARPSCAN:
+            return launch_warpscan(src, dst, n, p, st);
+        case BO_PS_TRANSPOSED: {
+            // row-wise [p][n] -> column-wise [n][p] in ws -> ACROSS in place -> back into dst
+            int rc = launch_transpose(src, ws, p, n, st);
+            if (rc) return rc;
+            rc = launch_across(static_cast<const T *>(ws), static_cast<T *>(ws), n, p, st);
+            if (rc) return rc;
+            return launch_transpose(ws, dst, n, p, st);
+        }
+        case BO_PS_NAIVE: {
+            const unsigned grid = static_cast<unsigned>((p + 63) / 64);
+            ps_naive<T><<<grid, 64, 0, st>>>(src, dst, n, p, layout);
+            return after_launch("ps_naive");
+        }
+        default:
+            return fail(BO_EINVAL, "prefix: unknown variant");
+    }
+}
+
+int prefix_dispatch(const void *src, void *dst, int64_t n, int64_t p, int dtype, int layout, int variant,
+                    void *ws, cudaStream_t st) {
+    if (dtype == BO_I32)
+        return run_prefix(static_cast<const int32_t *>(src), static_cast<int32_t *>(dst), n, p, layout,
+                          variant, ws, st);
+    return run_prefix(static_cast<const float *>(src), static_cast<float *>(dst), n, p, layout, variant, ws,
+                      st);
+}
+
+}  // namespace bo

@@ -1,0 +1,147 @@
+// transpose.cu -- row-wise <-> column-wise arrangement (Fig. 5):
+//     dst[c*rows + r] = src[r*cols + c]      (4-byte elements)
+//
+// Main kernel: persistent CTAs, TMA (cp.async.bulk.tensor) loads of
+// [64 rows x 32 cols] boxes with 128-byte swizzle into a STAGES-deep smem ring
+// (mbarrier complete_tx), a bank-conflict-free in-smem transpose (one 128-bit
+// swizzled read + four 32-bit swizzled writes per thread per sub-tile), and
+// TMA stores of two [32 x 32] boxes.  One __syncthreads per tile.
+// Fallback (unaligned shapes): classic padded [32][33] smem tile.
+#include "common.cuh"
+
+namespace bo {
+
+namespace tr {
+constexpr int kCols = 32;                      // box inner extent (128 B)
+constexpr int kRows = 64;                      // box outer extent (2 sub-tiles)
+constexpr int kStages = 6;
+constexpr int kOut = 2;
+constexpr int kThreads = 256;
+constexpr uint32_t kBoxBytes = kRows * kCols * 4;   // 8 KiB
+constexpr size_t kSmem = 1024 /*align slack*/ + (kStages + kOut) * kBoxBytes + kStages * 8;
+}  // namespace tr
+
+__global__ void __launch_bounds__(tr::kThreads)
+transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
+                     const __grid_constant__ CUtensorMap dst_map, int tiles_c, long long ntiles) {
+    using namespace tr;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *base = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                                ~uintptr_t(1023));
+    uint8_t *in_buf = base;                                   // kStages boxes
+    uint8_t *out_buf = base + kStages * kBoxBytes;            // kOut boxes (2 sub-tiles each)
+    uint64_t *full = reinterpret_cast<uint64_t *>(out_buf + kOut * kBoxBytes);
+
+    const int tid = threadIdx.x;
+    const int warp = tid >> 5, lane = tid & 31;
+    const long long first = blockIdx.x;
+    const long long count = ntiles > first ? (ntiles - 1 - first) / gridDim.x + 1 : 0;
+
+    if (tid == 0) {
+        prefetch_tmap(&src_map);
+        prefetch_tmap(&dst_map);
+        for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
+        fence_barrier_init();
+    }
+    __syncthreads();
+
+    auto issue_load = [&](long long i) {
+        const long long t = first + i * gridDim.x;
+        const int tc = static_cast<int>(t % tiles_c), trow = static_cast<int>(t / tiles_c);
+        const int s = static_cast<int>(i % kStages);
+        mbar_arrive_expect_tx(&full[s], kBoxBytes);
+        tma_load_2d(in_buf + s * kBoxBytes, &src_map, tc * kCols, trow * kRows, &full[s]);
+    };
+    if (tid == 0)
+        for (long long i = 0; i < count && i < kStages; ++i) issue_load(i);
+
+    for (long long i = 0; i < count; ++i) {
+        const int s = static_cast<int>(i % kStages);
+        const uint32_t ph = static_cast<uint32_t>((i / kStages) & 1);
+        uint8_t *ob = out_buf + (i % kOut) * kBoxBytes;
+        mbar_wait(&full[s], ph);
+        const uint8_t *ib = in_buf + s * kBoxBytes;
+#pragma unroll
+        for (int sub = 0; sub < kRows / 32; ++sub) {
+            const int r = sub * 32 + lane;                     // source row in box
+            const uint4 v = *reinterpret_cast<const uint4 *>(ib + swz128(r, warp));
+            uint8_t *os = ob + sub * (32 * 128);               // [32 cols][32 rows] sub-tile
+            const uint32_t vv[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int c = warp * 4 + q;                    // source col = dst row
+                *reinterpret_cast<uint32_t *>(os + swz128(c, lane >> 2) + (lane & 3) * 4) = vv[q];
+            }
+        }
+        fence_proxy_async_smem();
+        if (tid == 0) bulk_wait_read<0>();   // store i-1 has finished reading its buffer
+        __syncthreads();
+        if (tid == 0) {
+            const long long t = first + i * gridDim.x;
+            const int tc = static_cast<int>(t % tiles_c), trow = static_cast<int>(t / tiles_c);
+#pragma unroll
+            for (int sub = 0; sub < kRows / 32; ++sub)
+                tma_store_2d(&dst_map, ob + sub * (32 * 128), trow * kRows + sub * 32, tc * kCols);
+            bulk_commit();
+            if (i + kStages < count) issue_load(i + kStages);
+        }
+    }
+    if (tid == 0) bulk_wait<0>();
+}
+
+// Fallback for shapes TMA cannot describe (unaligned pointers, odd strides).
+__global__ void __launch_bounds__(256)
+transpose_smem_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, long long rows,
+                      long long cols, long long tiles_c, long long ntiles) {
+    __shared__ uint32_t tile[32][33];
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;   // 32 x 8
+    for (long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const long long r0 = (t / tiles_c) * 32, c0 = (t % tiles_c) * 32;
+#pragma unroll
+        for (int k = 0; k < 32; k += 8) {
+            const long long r = r0 + ty + k, c = c0 + tx;
+            if (r < rows && c < cols) tile[ty + k][tx] = src[r * cols + c];
+        }
+        __syncthreads();
+#pragma unroll
+        for (int k = 0; k < 32; k += 8) {
+            const long long c = c0 + ty + k, r = r0 + tx;
+            if (r < rows && c < cols) dst[c * rows + r] = tile[tx][ty + k];
+        }
+        __syncthreads();
+    }
+}
+
+bool transpose_tma_ok(const void *src, const void *dst, int64_t rows, int64_t cols) {
+    return aligned16(src) && aligned16(dst) && (cols % 4) == 0 && (rows % 4) == 0 &&
+           rows < (int64_t(1) << 31) && cols < (int64_t(1) << 31);
+}
+
+int launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, cudaStream_t st) {
+    if (rows == 0 || cols == 0) return BO_OK;
+    if (transpose_tma_ok(src, dst, rows, cols)) {
+        CUtensorMap smap, dmap;
+        if (!make_tmap_2d(&smap, src, rows, cols, tr::kRows, tr::kCols, CU_TENSOR_MAP_SWIZZLE_128B) ||
+            !make_tmap_2d(&dmap, dst, cols, rows, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B))
+            return fail(BO_ECUDA, "transpose: cuTensorMapEncodeTiled failed");
+        static bool attr = [] {
+            return cudaFuncSetAttribute(transpose_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        static_cast<int>(tr::kSmem)) == cudaSuccess;
+        }();
+        if (!attr) return fail(BO_ECUDA, "transpose: cannot set dynamic smem");
+        const long long tiles_c = (cols + tr::kCols - 1) / tr::kCols;
+        const long long tiles_r = (rows + tr::kRows - 1) / tr::kRows;
+        const long long ntiles = tiles_c * tiles_r;
+        const long long grid = std::min<long long>(ntiles, 3LL * num_sms());
+        transpose_tma_kernel<<<static_cast<unsigned>(grid), tr::kThreads, tr::kSmem, st>>>(
+            smap, dmap, static_cast<int>(tiles_c), ntiles);
+        return after_launch("transpose_tma_kernel");
+    }
+    const long long tiles_c = (cols + 31) / 32, ntiles = tiles_c * ((rows + 31) / 32);
+    const long long grid = std::min<long long>(ntiles, 16LL * num_sms());
+    transpose_smem_kernel<<<static_cast<unsigned>(grid), 256, 0, st>>>(
+        static_cast<const uint32_t *>(src), static_cast<uint32_t *>(dst), rows, cols, tiles_c, ntiles);
+    return after_launch("transpose_smem_kernel");
+}
+
+}  // namespace bo

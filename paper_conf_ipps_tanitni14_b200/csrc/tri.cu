@@ -1,0 +1,263 @@
+// tri.cu -- bulk optimal convex-polygon triangulation (Algorithm OPT,
+// P:174-200; Parallel Algorithm OPT).
+//
+// Per instance h, with M[i,i] = 0:
+//     M[i,j] = min_{k=i..j-1} (M[i,k] + M[k+1,j]) + c[i-1,j],   out[h] = M[1,n-1].
+// Cell (i,j) needs only cells of smaller j-i, so ANY topological order --
+// in particular the diagonal wavefront d = j-i = 1..n-2 -- gives the same
+// values, and because min is exact and every sum keeps its association
+// ((M[i,k] + M[k+1,j]) then + c), the k order of the min is free: results are
+// bit-identical to the sequential algorithm for int32 and for finite fp32.
+//
+//   THREAD_REG  thread per instance, whole table in registers (fully unrolled,
+//               n a template parameter, 3 <= n <= 18).
+//   UMM_GLOBAL  the paper's kernel: thread per instance, M in global memory
+//               in the same arrangement as c (row-wise (n-1)^2 h + ..., or
+//               column-wise interleaved cell*p + h), 64-thread
+//               blocks, one 32-bit access per step.
+//   SMEM_WARP   warp per instance, M in shared memory (row stride SP = 1 mod
+//               32 so diagonal-parallel row AND column reads are
+//               bank-conflict-free), diagonal wavefront, long diagonals split
+//               the k range over g lanes + xor-shuffle min.
+//   TILED       (tri_tiled.cu) warp per instance, 4x4 register tiles.
+#include "common.cuh"
+
+#include <climits>
+
+namespace bo {
+
+template <typename T>
+struct MinPlus;
+template <>
+struct MinPlus<int32_t> {
+    __host__ __device__ static constexpr int32_t inf() { return INT32_MAX; }
+    // min(a + b, s): one VIADDMNMX on sm_100a
+    static __device__ __forceinline__ int32_t addmin(int32_t a, int32_t b, int32_t s) {
+        return __viaddmin_s32(a, b, s);
+    }
+    static __device__ __forceinline__ int32_t add(int32_t a, int32_t b) { return add_wrap(a, b); }
+    static __device__ __forceinline__ int32_t min(int32_t a, int32_t b) { return ::min(a, b); }
+};
+template <>
+struct MinPlus<float> {
+    __host__ __device__ static constexpr float inf() { return __builtin_huge_valf(); }
+    static __device__ __forceinline__ float addmin(float a, float b, float s) {
+        return fminf(__fadd_rn(a, b), s);
+    }
+    static __device__ __forceinline__ float add(float a, float b) { return __fadd_rn(a, b); }
+    static __device__ __forceinline__ float min(float a, float b) { return fminf(a, b); }
+};
+
+__host__ __device__ __forceinline__ long long c_index(int layout, long long h, long long n, long long p,
+                                                      long long a, long long b) {
+    const long long e = a * n + b;
+    return layout == BO_ROW_WISE ? h * n * n + e : e * p + h;
+}
+
+// -------------------------------------------------------------- THREAD_REG
+template <typename T, int N>
+__global__ void __launch_bounds__(128)
+tri_thread_reg(const T *__restrict__ c, T *__restrict__ out, long long p, int layout) {
+    using Op = MinPlus<T>;
+    const long long h = blockIdx.x * 128LL + threadIdx.x;
+    if (h >= p) return;
+    T M[N][N];                         // 1-based M[i][j], i <= j; all indices compile-time
+#pragma unroll
+    for (int i = 1; i <= N - 1; ++i) M[i][i] = T(0);
+#pragma unroll
+    for (int i = N - 2; i >= 1; --i) {
+#pragma unroll
+        for (int j = i + 1; j <= N - 1; ++j) {
+            T s = Op::inf();
+#pragma unroll
+            for (int k = i; k <= j - 1; ++k) s = Op::addmin(M[i][k], M[k + 1][j], s);
+            M[i][j] = Op::add(s, __ldg(c + c_index(layout, h, N, p, i - 1, j)));
+        }
+    }
+    out[h] = M[1][N - 1];
+}
+
+// -------------------------------------------------------------- UMM_GLOBAL
+template <typename T>
+__global__ void __launch_bounds__(64)
+tri_umm_global(const T *__restrict__ c, T *__restrict__ out, T *M, long long n, long long p, int layout) {
+    const long long h = blockIdx.x * 64LL + threadIdx.x;
+    if (h >= p) return;
+    const long long n1 = n - 1;
+    auto mi = [&](long long i, long long j) -> long long {
+        const long long cell = (i - 1) * n1 + (j - 1);
+        return layout == BO_ROW_WISE ? h * n1 * n1 + cell : cell * p + h;
+    };
+    for (long long i = 1; i <= n - 1; ++i) M[mi(i, i)] = T(0);
+    for (long long i = n - 2; i >= 1; --i) {
+        for (long long j = i + 1; j <= n - 1; ++j) {
+            T s = MinPlus<T>::inf();
+            for (long long k = i; k <= j - 1; ++k) {
+                const T r = MinPlus<T>::add(M[mi(i, k)], M[mi(k + 1, j)]);
+                s = r < s ? r : s;
+            }
+            M[mi(i, j)] = MinPlus<T>::add(s, c[c_index(layout, h, n, p, i - 1, j)]);
+        }
+    }
+    out[h] = M[mi(1, n - 1)];
+}
+
+// --------------------------------------------------------------- SMEM_WARP
+// Table S (0-based a = i-1, b = j-1), row stride SP: S[a*SP + b] = M[a+1][b+1]
+// for b >= a; before cell (a,b) is computed it holds c[a][b+1].
+template <typename T>
+__global__ void __launch_bounds__(512)
+tri_smem_warp(const T *__restrict__ c, T *__restrict__ out, int n, long long p, int layout, int SP, int W) {
+    using Op = MinPlus<T>;
+    extern __shared__ uint8_t smem_raw[];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int n1 = n - 1;
+    T *S = reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warp) * n1 * SP;
+    const int cells = n1 * n1;
+
+    for (long long hb = static_cast<long long>(blockIdx.x) * W; hb < p; hb += static_cast<long long>(gridDim.x) * W) {
+        const long long h = hb + warp;
+        if (layout == BO_ROW_WISE) {
+            if (h < p) {
+                const T *ch = c + h * n * n;
+                for (int a = 0; a < n1; ++a)
+                    for (int b = a + lane; b < n1; b += 32)
+                        S[a * SP + b] = b == a ? T(0) : __ldg(ch + a * n + b + 1);
+            }
+        } else {
+            // column-wise c[(a*n+b)*p + h]: consecutive threads take consecutive
+            // instances of the CTA so every 32-byte sector is fully used.
+            __syncthreads();
+            T *S0 = reinterpret_cast<T *>(smem_raw);
+            for (int f = tid; f < W * cells; f += blockDim.x) {
+                const int w = f % W, cell = f / W;
+                const int a = cell / n1, b = cell % n1;
+                if (b < a || hb + w >= p) continue;
+                S0[static_cast<size_t>(w) * n1 * SP + a * SP + b] =
+                    b == a ? T(0) : __ldg(c + (static_cast<long long>(a) * n + b + 1) * p + hb + w);
+            }
+            __syncthreads();
+        }
+        __syncwarp();
+        if (h < p) {
+            for (int d = 1; d <= n - 2; ++d) {
+                const int C = n1 - d;                     // cells (a, a+d), a = 0..C-1
+                int g = 1;
+                while (g < 32 && C * g * 2 <= 32) g <<= 1;   // k split factor
+                const int per = 32 / g;
+                for (int cb = 0; cb < C; cb += per) {
+                    const int a = cb + lane / g, q = lane % g;
+                    const int b = a + d;
+                    T s = Op::inf();
+                    if (a < C) {
+                        const T *row = S + a * SP;
+                        for (int k = a + q; k <= b - 1; k += g) s = Op::addmin(row[k], S[(k + 1) * SP + b], s);
+                    }
+                    for (int off = 1; off < g; off <<= 1) s = Op::min(s, __shfl_xor_sync(0xffffffffu, s, off));
+                    if (a < C && q == 0) S[a * SP + b] = Op::add(s, S[a * SP + b]);
+                }
+                __syncwarp();
+            }
+            if (lane == 0) out[h] = S[n - 2];
+        }
+        __syncwarp();
+    }
+}
+
+// ------------------------------------------------------------------- host
+int tiled_supported(int64_t n);
+int launch_tri_tiled(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, cudaStream_t st);
+
+static int smem_sp(int64_t n) {
+    const int n1 = static_cast<int>(n - 1);
+    return ((n1 - 1 + 31) / 32) * 32 + 1;   // >= n1, == 1 mod 32
+}
+
+static size_t smem_per_instance(int64_t n) { return static_cast<size_t>(n - 1) * smem_sp(n) * 4; }
+
+int resolve_tri_variant(int64_t n, int64_t p, int dtype, int layout, int variant) {
+    (void)p; (void)dtype; (void)layout;
+    if (variant != BO_AUTO) return variant;
+    if (n <= 16) return BO_TRI_THREAD_REG;
+    if (tiled_supported(n)) return BO_TRI_TILED;
+    if (smem_per_instance(n) <= 200 * 1024) return BO_TRI_SMEM_WARP;
+    return BO_TRI_UMM_GLOBAL;
+}
+
+size_t tri_workspace(int64_t n, int64_t p, int variant) {
+    if (variant == BO_TRI_UMM_GLOBAL) return static_cast<size_t>(n - 1) * (n - 1) * p * 4;
+    return 0;
+}
+
+template <typename T, int N>
+static int launch_reg_n(const void *c, void *out, int64_t p, int layout, cudaStream_t st) {
+    const unsigned grid = static_cast<unsigned>((p + 127) / 128);
+    tri_thread_reg<T, N><<<grid, 128, 0, st>>>(static_cast<const T *>(c), static_cast<T *>(out), p, layout);
+    return after_launch("tri_thread_reg");
+}
+
+template <typename T>
+static int launch_reg(const void *c, void *out, int64_t n, int64_t p, int layout, cudaStream_t st) {
+    switch (n) {
+#define BO_REG_CASE(N) \
+    case N: return launch_reg_n<T, N>(c, out, p, layout, st);
+        BO_REG_CASE(3) BO_REG_CASE(4) BO_REG_CASE(5) BO_REG_CASE(6) BO_REG_CASE(7) BO_REG_CASE(8)
+        BO_REG_CASE(9) BO_REG_CASE(10) BO_REG_CASE(11) BO_REG_CASE(12) BO_REG_CASE(13) BO_REG_CASE(14)
+        BO_REG_CASE(15) BO_REG_CASE(16) BO_REG_CASE(17) BO_REG_CASE(18)
+#undef BO_REG_CASE
+        default:
+            return fail(BO_EUNSUPPORTED, "triangulation THREAD_REG supports 3 <= n <= 18");
+    }
+}
+
+template <typename T>
+static int launch_smem_warp(const void *c, void *out, int64_t n, int64_t p, int layout, cudaStream_t st) {
+    const size_t per = smem_per_instance(n);
+    if (per > 200 * 1024) return fail(BO_EUNSUPPORTED, "triangulation SMEM_WARP: table does not fit in smem");
+    static bool attr = [] {
+        return cudaFuncSetAttribute(tri_smem_warp<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024) ==
+               cudaSuccess;
+    }();
+    if (!attr) return fail(BO_ECUDA, "triangulation SMEM_WARP: cannot set dynamic smem");
+    // warps per CTA: as many instances as fit in one SM's smem, at most 16
+    int W = static_cast<int>(std::min<size_t>(16, (227 * 1024) / per));
+    W = std::max(W, 1);
+    const size_t smem = W * per;
+    int per_sm = 1;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_smem_warp<T>, W * 32, smem);
+    per_sm = std::max(per_sm, 1);
+    const long long blocks = std::min<long long>((p + W - 1) / W, static_cast<long long>(per_sm) * num_sms() * 8);
+    tri_smem_warp<T><<<static_cast<unsigned>(blocks), W * 32, smem, st>>>(
+        static_cast<const T *>(c), static_cast<T *>(out), static_cast<int>(n), p, layout, smem_sp(n), W);
+    return after_launch("tri_smem_warp");
+}
+
+template <typename T>
+static int run_tri(const void *c, void *out, int64_t n, int64_t p, int layout, int variant, void *ws,
+                   cudaStream_t st) {
+    switch (variant) {
+        case BO_TRI_THREAD_REG:
+            return launch_reg<T>(c, out, n, p, layout, st);
+        case BO_TRI_UMM_GLOBAL: {
+            const unsigned grid = static_cast<unsigned>((p + 63) / 64);
+            tri_umm_global<T><<<grid, 64, 0, st>>>(static_cast<const T *>(c), static_cast<T *>(out),
+                                                   static_cast<T *>(ws), n, p, layout);
+            return after_launch("tri_umm_global");
+        }
+        case BO_TRI_SMEM_WARP:
+            return launch_smem_warp<T>(c, out, n, p, layout, st);
+        case BO_TRI_TILED:
+            if (!tiled_supported(n)) return fail(BO_EUNSUPPORTED, "triangulation TILED supports 5 <= n <= 64");
+            return launch_tri_tiled(c, out, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout, st);
+        default:
+            return fail(BO_EINVAL, "triangulation: unknown variant");
+    }
+}
+
+int tri_dispatch(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int variant, void *ws,
+                 cudaStream_t st) {
+    if (dtype == BO_I32) return run_tri<int32_t>(c, out, n, p, layout, variant, ws, st);
+    return run_tri<float>(c, out, n, p, layout, variant, ws, st);
+}
+
+}  // namespace bo

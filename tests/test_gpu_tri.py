@@ -1,0 +1,112 @@
+"""GPU parity: bulk optimal triangulation (every variant, both layouts, both
+dtypes) against the CPU oracle -- bit-exact (min is exact and each sum keeps
+the association of Algorithm OPT).  Full TR-1 and TR-2 configs
+are verified on every instance."""
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import bulkgen
+import oracle
+import paper_conf_ipps_tanitni14_b200 as bo
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda"
+NTHREADS = os.cpu_count() or 1
+
+
+def _variants(n):
+    v = [bo.AUTO, bo.TRI_UMM_GLOBAL, bo.TRI_SMEM_WARP]
+    if n <= 18:
+        v.append(bo.TRI_THREAD_REG)
+    if bo.triangulation_variant(n, 1, bo.F32, bo.ROW_WISE, bo.AUTO) == bo.TRI_TILED or 5 <= n <= 64:
+        v.append(bo.TRI_TILED)
+    return v
+
+
+def _supported(n, variant):
+    if variant == bo.TRI_TILED:
+        try:
+            bo.triangulation(torch.zeros((1, n, n), device=DEV), bo.ROW_WISE, bo.TRI_TILED)
+        except bo.BulkError as e:
+            if e.status == -2:
+                return False
+            raise
+    return True
+
+
+CASES = [(3, 5), (4, 33), (5, 64), (8, 100), (13, 257), (16, 300), (17, 64), (18, 40), (24, 100), (33, 64),
+         (40, 70), (63, 33), (64, 130), (65, 20), (100, 9), (128, 4)]
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("n,p", CASES)
+def test_all_variants_match_oracle(dt, layout, n, p):
+    c = bulkgen.tri_input(n, p, seed=n + 100 * p, dtype=dt, layout=layout)
+    ref = oracle.bulk_opt(c, layout, nthreads=NTHREADS)
+    ct = torch.from_numpy(c).to(DEV)
+    for v in _variants(n):
+        if not _supported(n, v):
+            continue
+        got = bo.triangulation(ct, layout, v).cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), (n, p, v)
+
+
+def test_n3_is_zero_and_closed_forms():
+    c = torch.zeros((10, 3, 3), dtype=torch.int32, device=DEV)
+    assert torch.all(bo.triangulation(c) == 0)
+    # uniform chord weight w -> (n-3) w for every n
+    for n in (5, 16, 17, 40, 64):
+        w = np.zeros((n, n), dtype=np.int32)
+        for a in range(n):
+            for b in range(a + 2, n):
+                if not (a == 0 and b == n - 1):
+                    w[a, b] = 5
+        ct = torch.from_numpy(np.broadcast_to(w, (7, n, n)).copy()).to(DEV)
+        for v in _variants(n):
+            if _supported(n, v):
+                assert torch.all(bo.triangulation(ct, bo.ROW_WISE, v) == (n - 3) * 5), (n, v)
+
+
+def test_hand_worked_pentagon():
+    c = np.zeros((5, 5), dtype=np.int32)
+    for (a, b), w in {(0, 2): 7, (0, 3): 2, (1, 3): 5, (1, 4): 9, (2, 4): 4}.items():
+        c[a, b] = w
+    got = bo.triangulation(torch.from_numpy(c[None]).to(DEV)).cpu().numpy()
+    assert got.tolist() == [7]      # tests/golden/pentagon_worked.txt
+
+
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+def test_tr1_full_config(layout):
+    n, p = 16, 65536
+    c = bo.generate_tri(n, p, 3, torch.int32, layout)
+    got = bo.triangulation(c, layout).cpu().numpy()
+    ref = oracle.bulk_opt(bulkgen.tri_input(n, p, 3, "int32", layout), layout, nthreads=NTHREADS)
+    assert np.array_equal(got, ref)
+
+
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+def test_tr2_full_config(layout):
+    n, p = 64, 65536
+    c = bo.generate_tri(n, p, 4, torch.float32, layout)
+    got = bo.triangulation(c, layout).cpu().numpy()
+    ids = np.arange(p) if NTHREADS >= 16 else np.unique(np.r_[np.arange(0, p, 16), p - 1])
+    ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 4, "float32"), oracle.ROW_WISE, nthreads=NTHREADS)
+    assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("variant", [bo.TRI_SMEM_WARP, bo.TRI_TILED, bo.TRI_UMM_GLOBAL])
+def test_tr2_variants_agree_full_size(variant):
+    n, p = 64, 65536
+    c = bo.generate_tri(n, p, 4, torch.float32, bo.ROW_WISE)
+    if not _supported(n, variant):
+        pytest.skip("variant not built")
+    a = bo.triangulation(c, bo.ROW_WISE, variant)
+    b = bo.triangulation(bo.transpose(c.view(p, n * n)).view(n, n, p), bo.COLUMN_WISE, variant)
+    assert torch.equal(a.view(torch.int32), b.view(torch.int32))
+    ids = np.arange(0, p, 997)
+    ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 4, "float32"), oracle.ROW_WISE, nthreads=NTHREADS)
+    assert np.array_equal(a.cpu().numpy()[ids].view(np.uint32), ref.view(np.uint32))
