@@ -76,8 +76,10 @@ typedef enum {
     BO_TRI_SMEM_WARP = 17,  /* warp per instance, M in shared memory, diagonal
                                wavefront, k split across lanes + shuffle min      */
     BO_TRI_THREAD_REG = 18, /* thread per instance, M in registers (3 <= n <= 18) */
-    BO_TRI_TILED = 19       /* warp per instance, M in shared memory, 4x4 register
-                               tiles (min-plus blocked product), n <= 64          */
+    BO_TRI_TILED = 19,      /* warp per instance, M in shared memory, 4x4 register
+                               tiles (min-plus blocked product), 5 <= n <= 64     */
+    BO_TRI_TILED_HALF = 20  /* as BO_TRI_TILED with 16 lanes per instance (two
+                               instances per warp)                                 */
 } bo_variant;
 
 /* ------------------------------------------------------------------------- */

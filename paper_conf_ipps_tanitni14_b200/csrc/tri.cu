@@ -77,6 +77,61 @@ tri_thread_reg(const T *__restrict__ c, T *__restrict__ out, long long p, int la
     out[h] = M[1][N - 1];
 }
 
+// THREAD_REG fed by TMA: a warp's 32 instances have their weights staged in
+// shared memory by cp.async.bulk.tensor boxes of [32 instances x 32
+// elements] (row-wise c: box = 32 consecutive elements of 32 instances,
+// 128B-swizzled, read back as conflict-free 128-bit chunks; column-wise c:
+// box = 32 elements x 32 consecutive instances, read back one word per lane).
+// Only the elements up to the last one Algorithm OPT reads are fetched.
+template <typename T, int N, int LAYOUT>
+__global__ void __launch_bounds__(32)
+tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out, long long p) {
+    using Op = MinPlus<T>;
+    constexpr int NE = (N - 3) * N + N;          // c[N-3][N-1] is the last weight read
+    constexpr int NB = (NE + 31) / 32;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint64_t *bar = reinterpret_cast<uint64_t *>(buf + NB * 4096);
+    const int t = threadIdx.x;
+    if (t == 0) {
+        prefetch_tmap(&cmap);
+        mbar_init(bar, 1);
+        fence_barrier_init();
+        mbar_arrive_expect_tx(bar, NB * 4096);
+#pragma unroll
+        for (int b = 0; b < NB; ++b) {
+            if (LAYOUT == BO_ROW_WISE) tma_load_2d(buf + b * 4096, &cmap, b * 32, blockIdx.x * 32, bar);
+            else tma_load_2d(buf + b * 4096, &cmap, blockIdx.x * 32, b * 32, bar);
+        }
+    }
+    __syncwarp();
+    mbar_wait(bar, 0);
+    auto cl = [&](int e) -> T {
+        const uint8_t *box = buf + (e >> 5) * 4096;
+        if (LAYOUT == BO_ROW_WISE) {
+            const uint4 v = *reinterpret_cast<const uint4 *>(box + swz128(t, (e & 31) >> 2));
+            const uint32_t w = (e & 3) == 0 ? v.x : (e & 3) == 1 ? v.y : (e & 3) == 2 ? v.z : v.w;
+            return *reinterpret_cast<const T *>(&w);
+        }
+        return *reinterpret_cast<const T *>(box + (e & 31) * 128 + t * 4);
+    };
+    T M[N][N];
+#pragma unroll
+    for (int i = 1; i <= N - 1; ++i) M[i][i] = T(0);
+#pragma unroll
+    for (int i = N - 2; i >= 1; --i) {
+#pragma unroll
+        for (int j = i + 1; j <= N - 1; ++j) {
+            T s = Op::inf();
+#pragma unroll
+            for (int k = i; k <= j - 1; ++k) s = Op::addmin(M[i][k], M[k + 1][j], s);
+            M[i][j] = Op::add(s, cl((i - 1) * N + j));
+        }
+    }
+    const long long h = blockIdx.x * 32LL + t;
+    if (h < p) out[h] = M[1][N - 1];
+}
+
 // -------------------------------------------------------------- UMM_GLOBAL
 template <typename T>
 __global__ void __launch_bounds__(64)
@@ -166,7 +221,8 @@ tri_smem_warp(const T *__restrict__ c, T *__restrict__ out, int n, long long p, 
 
 // ------------------------------------------------------------------- host
 int tiled_supported(int64_t n);
-int launch_tri_tiled(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, cudaStream_t st);
+int launch_tri_tiled(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int lpi,
+                     cudaStream_t st);
 
 static int smem_sp(int64_t n) {
     const int n1 = static_cast<int>(n - 1);
@@ -189,8 +245,32 @@ size_t tri_workspace(int64_t n, int64_t p, int variant) {
     return 0;
 }
 
+template <typename T, int N, int LAYOUT>
+static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) {
+    constexpr int NE = (N - 3) * N + N;
+    constexpr int NB = (NE + 31) / 32;
+    constexpr size_t smem = 1024 + NB * 4096 + 16;
+    CUtensorMap map;
+    const bool ok = LAYOUT == BO_ROW_WISE
+                        ? make_tmap_2d(&map, c, p, N * N, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
+                        : make_tmap_2d(&map, c, N * N, p, 32, 32, CU_TENSOR_MAP_SWIZZLE_NONE);
+    if (!ok) return fail(BO_ECUDA, "triangulation THREAD_REG: cuTensorMapEncodeTiled failed");
+    static bool attr = [] {
+        return cudaFuncSetAttribute(tri_thread_reg_tma<T, N, LAYOUT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    static_cast<int>(smem)) == cudaSuccess;
+    }();
+    if (!attr) return fail(BO_ECUDA, "triangulation THREAD_REG: cannot set dynamic smem");
+    const unsigned grid = static_cast<unsigned>((p + 31) / 32);
+    tri_thread_reg_tma<T, N, LAYOUT><<<grid, 32, smem, st>>>(map, static_cast<T *>(out), p);
+    return after_launch("tri_thread_reg_tma");
+}
+
 template <typename T, int N>
 static int launch_reg_n(const void *c, void *out, int64_t p, int layout, cudaStream_t st) {
+    if (p >= 32 && N >= 6 && p < (int64_t(1) << 31) && aligned16(c)) {
+        if (layout == BO_ROW_WISE && (N * N) % 4 == 0) return launch_reg_tma<T, N, BO_ROW_WISE>(c, out, p, st);
+        // column-wise c is already coalesced for thread-per-instance: direct loads win (measured)
+    }
     const unsigned grid = static_cast<unsigned>((p + 127) / 128);
     tri_thread_reg<T, N><<<grid, 128, 0, st>>>(static_cast<const T *>(c), static_cast<T *>(out), p, layout);
     return after_launch("tri_thread_reg");
@@ -247,8 +327,10 @@ static int run_tri(const void *c, void *out, int64_t n, int64_t p, int layout, i
         case BO_TRI_SMEM_WARP:
             return launch_smem_warp<T>(c, out, n, p, layout, st);
         case BO_TRI_TILED:
+        case BO_TRI_TILED_HALF:
             if (!tiled_supported(n)) return fail(BO_EUNSUPPORTED, "triangulation TILED supports 5 <= n <= 64");
-            return launch_tri_tiled(c, out, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout, st);
+            return launch_tri_tiled(c, out, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout,
+                                    variant == BO_TRI_TILED ? 32 : 16, st);
         default:
             return fail(BO_EINVAL, "triangulation: unknown variant");
     }
