@@ -115,6 +115,35 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// ---------------------------------------------------------------- work queue
+// Dynamic tile scheduler for persistent kernels: CTA b starts on tile b, then
+// claims gridDim.x + (ticket) until the tiles run out, so SMs that run faster
+// (L2 die, DRAM channel mix) take more tiles.  The last CTA to retire resets
+// the slot, so no host memset is needed between launches; the host rotates
+// through kWorkSlots slots so launches on different streams do not share one.
+struct WorkSlot {
+    unsigned long long next;
+    unsigned int done;
+    unsigned int pad;
+};
+constexpr int kWorkSlots = 256;
+
+__device__ __forceinline__ long long claim_tile(WorkSlot *w) {
+    return static_cast<long long>(gridDim.x) + static_cast<long long>(atomicAdd(&w->next, 1ull));
+}
+__device__ __forceinline__ void retire_cta(WorkSlot *w) {
+    __threadfence();
+    if (atomicAdd(&w->done, 1u) == gridDim.x - 1) {
+        w->next = 0;
+        w->done = 0;
+        __threadfence();
+    }
+}
+
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
 }

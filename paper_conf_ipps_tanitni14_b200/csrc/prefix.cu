@@ -96,22 +96,24 @@ constexpr int kInst = 128;                 // instances per tile = threads per C
 constexpr int kElems = 32;                 // elements per chunk (128 B rows, swizzle 128B)
 constexpr int kStages = 6;
 constexpr uint32_t kBoxBytes = kInst * kElems * 4;   // 16 KiB
-constexpr size_t kSmem = 1024 + kStages * kBoxBytes + kStages * 8;
+constexpr size_t kSmem = 1024 + kStages * kBoxBytes + kStages * 16;
 }  // namespace fr
+
+__device__ WorkSlot g_fr_slots[kWorkSlots];
 
 template <typename T>
 __global__ void __launch_bounds__(fr::kInst)
 ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant__ CUtensorMap dst_map,
-                 long long ntiles, int nchunks) {
+                 long long ntiles, int nchunks, int slot) {
     using namespace fr;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                                ~uintptr_t(1023));
     uint64_t *full = reinterpret_cast<uint64_t *>(buf + kStages * kBoxBytes);
+    int *stage_tile = reinterpret_cast<int *>(full + kStages);    // tile of each ring slot, -1 = end
+    int *stage_chunk = stage_tile + kStages;
+    WorkSlot *ws = &g_fr_slots[slot];
     const int tid = threadIdx.x;
-    const long long first = blockIdx.x;
-    const long long my_tiles = ntiles > first ? (ntiles - 1 - first) / gridDim.x + 1 : 0;
-    const long long items = my_tiles * nchunks;
 
     if (tid == 0) {
         prefetch_tmap(&src_map);
@@ -121,26 +123,39 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
     }
     __syncthreads();
 
-    auto coords = [&](long long i, int &c0, int &c1) {
-        const long long tile = first + (i / nchunks) * gridDim.x;
-        c0 = static_cast<int>(i % nchunks) * kElems;
-        c1 = static_cast<int>(tile * kInst);
-    };
-    auto issue_load = [&](long long i) {
-        int c0, c1;
-        coords(i, c0, c1);
-        const int s = static_cast<int>(i % kStages);
+    // producer state (thread 0 only): next (tile, chunk) to load
+    long long prod_tile = blockIdx.x;
+    int prod_chunk = 0;
+    bool prod_done = false;
+    auto issue = [&](int s) {
+        if (prod_chunk == nchunks) {
+            prod_tile = claim_tile(ws);
+            prod_chunk = 0;
+        }
+        if (prod_tile >= ntiles) {
+            stage_tile[s] = -1;
+            prod_done = true;
+            mbar_arrive(&full[s]);
+            return;
+        }
+        stage_tile[s] = static_cast<int>(prod_tile);
+        stage_chunk[s] = prod_chunk;
         mbar_arrive_expect_tx(&full[s], kBoxBytes);
-        tma_load_2d(buf + s * kBoxBytes, &src_map, c0, c1, &full[s]);
+        tma_load_2d(buf + s * kBoxBytes, &src_map, prod_chunk * kElems, static_cast<int>(prod_tile * kInst),
+                    &full[s]);
+        ++prod_chunk;
     };
     if (tid == 0)
-        for (long long i = 0; i < items && i < kStages - 1; ++i) issue_load(i);
+        for (int s = 0; s < kStages - 1 && !prod_done; ++s) issue(s);
 
     T r = T(0);
-    for (long long i = 0; i < items; ++i) {
+    for (long long i = 0;; ++i) {
         const int s = static_cast<int>(i % kStages);
-        if (i % nchunks == 0) r = T(0);                 // new tile: r_j <- 0
         mbar_wait(&full[s], static_cast<uint32_t>((i / kStages) & 1));
+        const int tile = stage_tile[s];
+        if (tile < 0) break;
+        const int chunk = stage_chunk[s];
+        if (chunk == 0) r = T(0);                       // new tile: r_j <- 0
         uint8_t *box = buf + s * kBoxBytes;
 #pragma unroll
         for (int k = 0; k < kElems / 4; ++k) {
@@ -155,15 +170,16 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
         fence_proxy_async_smem();
         __syncthreads();
         if (tid == 0) {
-            int c0, c1;
-            coords(i, c0, c1);
-            tma_store_2d(&dst_map, box, c0, c1);
+            tma_store_2d(&dst_map, box, chunk * kElems, tile * kInst);
             bulk_commit();
             bulk_wait_read<1>();                       // store i-1 no longer reads its stage
-            if (i + kStages - 1 < items) issue_load(i + kStages - 1);
+            if (!prod_done) issue(static_cast<int>((i + kStages - 1) % kStages));
         }
     }
-    if (tid == 0) bulk_wait<0>();
+    if (tid == 0) {
+        bulk_wait<0>();
+        retire_cta(ws);
+    }
 }
 
 // Fallback for any n / alignment: coalesced warp loads into a padded tile.
@@ -301,8 +317,10 @@ static int launch_fused_row(const T *src, T *dst, int64_t n, int64_t p, cudaStre
         const long long ntiles = (p + fr::kInst - 1) / fr::kInst;
         const int nchunks = static_cast<int>((n + fr::kElems - 1) / fr::kElems);
         const long long grid = std::min<long long>(ntiles, 2LL * num_sms());
+        static std::atomic<unsigned> next_slot{0};
+        const int slot = static_cast<int>(next_slot.fetch_add(1) % kWorkSlots);
         ps_fused_row_tma<T><<<static_cast<unsigned>(grid), fr::kInst, fr::kSmem, st>>>(smap, dmap, ntiles,
-                                                                                     nchunks);
+                                                                                     nchunks, slot);
         return after_launch("ps_fused_row_tma");
     }
     const long long blocks = std::min<long long>((p + 127) / 128, 16LL * num_sms());

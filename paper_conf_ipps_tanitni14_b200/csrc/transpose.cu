@@ -18,12 +18,14 @@ constexpr int kStages = 6;
 constexpr int kOut = 2;
 constexpr int kThreads = 256;
 constexpr uint32_t kBoxBytes = kRows * kCols * 4;   // 8 KiB
-constexpr size_t kSmem = 1024 /*align slack*/ + (kStages + kOut) * kBoxBytes + kStages * 8;
+constexpr size_t kSmem = 1024 /*align slack*/ + (kStages + kOut) * kBoxBytes + kStages * 16;
 }  // namespace tr
+
+__device__ WorkSlot g_tr_slots[kWorkSlots];
 
 __global__ void __launch_bounds__(tr::kThreads)
 transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
-                     const __grid_constant__ CUtensorMap dst_map, int tiles_c, long long ntiles) {
+                     const __grid_constant__ CUtensorMap dst_map, int tiles_c, long long ntiles, int slot) {
     using namespace tr;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *base = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -31,11 +33,11 @@ transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
     uint8_t *in_buf = base;                                   // kStages boxes
     uint8_t *out_buf = base + kStages * kBoxBytes;            // kOut boxes (2 sub-tiles each)
     uint64_t *full = reinterpret_cast<uint64_t *>(out_buf + kOut * kBoxBytes);
+    long long *stage_tile = reinterpret_cast<long long *>(full + kStages);   // -1 = end
+    WorkSlot *ws = &g_tr_slots[slot];
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
-    const long long first = blockIdx.x;
-    const long long count = ntiles > first ? (ntiles - 1 - first) / gridDim.x + 1 : 0;
 
     if (tid == 0) {
         prefetch_tmap(&src_map);
@@ -45,21 +47,32 @@ transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
     }
     __syncthreads();
 
-    auto issue_load = [&](long long i) {
-        const long long t = first + i * gridDim.x;
+    long long next_tile = blockIdx.x;        // producer state (thread 0)
+    bool prod_done = false;
+    auto issue = [&](int s) {
+        const long long t = next_tile;
+        if (t >= ntiles) {
+            stage_tile[s] = -1;
+            prod_done = true;
+            mbar_arrive(&full[s]);
+            return;
+        }
+        next_tile = claim_tile(ws);
+        stage_tile[s] = t;
         const int tc = static_cast<int>(t % tiles_c), trow = static_cast<int>(t / tiles_c);
-        const int s = static_cast<int>(i % kStages);
         mbar_arrive_expect_tx(&full[s], kBoxBytes);
         tma_load_2d(in_buf + s * kBoxBytes, &src_map, tc * kCols, trow * kRows, &full[s]);
     };
     if (tid == 0)
-        for (long long i = 0; i < count && i < kStages; ++i) issue_load(i);
+        for (int s = 0; s < kStages && !prod_done; ++s) issue(s);
 
-    for (long long i = 0; i < count; ++i) {
+    for (long long i = 0;; ++i) {
         const int s = static_cast<int>(i % kStages);
         const uint32_t ph = static_cast<uint32_t>((i / kStages) & 1);
         uint8_t *ob = out_buf + (i % kOut) * kBoxBytes;
         mbar_wait(&full[s], ph);
+        const long long t = stage_tile[s];
+        if (t < 0) break;
         const uint8_t *ib = in_buf + s * kBoxBytes;
 #pragma unroll
         for (int sub = 0; sub < kRows / 32; ++sub) {
@@ -77,16 +90,18 @@ transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
         if (tid == 0) bulk_wait_read<0>();   // store i-1 has finished reading its buffer
         __syncthreads();
         if (tid == 0) {
-            const long long t = first + i * gridDim.x;
             const int tc = static_cast<int>(t % tiles_c), trow = static_cast<int>(t / tiles_c);
 #pragma unroll
             for (int sub = 0; sub < kRows / 32; ++sub)
                 tma_store_2d(&dst_map, ob + sub * (32 * 128), trow * kRows + sub * 32, tc * kCols);
             bulk_commit();
-            if (i + kStages < count) issue_load(i + kStages);
+            if (!prod_done) issue(s);        // every thread has finished reading in[s]
         }
     }
-    if (tid == 0) bulk_wait<0>();
+    if (tid == 0) {
+        bulk_wait<0>();
+        retire_cta(ws);
+    }
 }
 
 // Fallback for shapes TMA cannot describe (unaligned pointers, odd strides).
@@ -133,8 +148,10 @@ int launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, cud
         const long long tiles_r = (rows + tr::kRows - 1) / tr::kRows;
         const long long ntiles = tiles_c * tiles_r;
         const long long grid = std::min<long long>(ntiles, 3LL * num_sms());
+        static std::atomic<unsigned> next_slot{0};
+        const int slot = static_cast<int>(next_slot.fetch_add(1) % kWorkSlots);
         transpose_tma_kernel<<<static_cast<unsigned>(grid), tr::kThreads, tr::kSmem, st>>>(
-            smap, dmap, static_cast<int>(tiles_c), ntiles);
+            smap, dmap, static_cast<int>(tiles_c), ntiles, slot);
         return after_launch("transpose_tma_kernel");
     }
     const long long tiles_c = (cols + 31) / 32, ntiles = tiles_c * ((rows + 31) / 32);
