@@ -92,20 +92,25 @@ ps_across_scalar(const T *src, T *dst, long long n, long long p) {
 
 // --------------------------------------------------------------- FUSED_ROW
 namespace fr {
-constexpr int kInst = 128;                 // instances per tile = threads per CTA
+// INST instances per tile = threads per CTA: 128 normally, 32 when p is so
+// small that 128-instance tiles would leave SMs idle (p < 2 * SMs * 128).
 constexpr int kElems = 32;                 // elements per chunk (128 B rows, swizzle 128B)
-constexpr int kStages = 6;
-constexpr uint32_t kBoxBytes = kInst * kElems * 4;   // 16 KiB
-constexpr size_t kSmem = 1024 + kStages * kBoxBytes + kStages * 16;
+template <int INST> struct Cfg {
+    static constexpr int kStages = INST == 128 ? 6 : 8;
+    static constexpr uint32_t kBoxBytes = INST * kElems * 4;   // 16 KiB / 4 KiB
+    static constexpr size_t kSmem = 1024 + kStages * kBoxBytes + kStages * 16;
+};
 }  // namespace fr
 
 __device__ WorkSlot g_fr_slots[kWorkSlots];
 
-template <typename T>
-__global__ void __launch_bounds__(fr::kInst)
+template <typename T, int kInst>
+__global__ void __launch_bounds__(kInst)
 ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant__ CUtensorMap dst_map,
                  long long ntiles, int nchunks, int slot) {
-    using namespace fr;
+    using fr::kElems;
+    constexpr int kStages = fr::Cfg<kInst>::kStages;
+    constexpr uint32_t kBoxBytes = fr::Cfg<kInst>::kBoxBytes;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                                ~uintptr_t(1023));
@@ -291,37 +296,48 @@ int resolve_prefix_variant(int64_t n, int64_t p, int layout, int variant, const 
 
 template <typename T>
 static int launch_across(const T *src, T *dst, int64_t n, int64_t p, cudaStream_t st) {
-    if (p % 4 == 0 && aligned16(src) && aligned16(dst)) {
+    // 128-bit lanes when there are enough instances to fill the GPU with
+    // 4-instance threads; otherwise one instance per thread, 16 rows in flight
+    if (p % 4 == 0 && aligned16(src) && aligned16(dst) && p / 4 >= 512LL * num_sms()) {
         const long long p4 = p / 4;
         const unsigned grid = static_cast<unsigned>((p4 + 255) / 256);
         ps_across_vec4<T, 8><<<grid, 256, 0, st>>>(src, dst, n, p4);
         return after_launch("ps_across_vec4");
     }
     const unsigned grid = static_cast<unsigned>((p + 255) / 256);
-    ps_across_scalar<T, 8><<<grid, 256, 0, st>>>(src, dst, n, p);
+    ps_across_scalar<T, 16><<<grid, 256, 0, st>>>(src, dst, n, p);
     return after_launch("ps_across_scalar");
+}
+
+template <typename T, int INST>
+static int launch_fused_row_tma(const T *src, T *dst, int64_t n, int64_t p, cudaStream_t st) {
+    using C = fr::Cfg<INST>;
+    CUtensorMap smap, dmap;
+    if (!make_tmap_2d(&smap, src, p, n, INST, fr::kElems, CU_TENSOR_MAP_SWIZZLE_128B) ||
+        !make_tmap_2d(&dmap, dst, p, n, INST, fr::kElems, CU_TENSOR_MAP_SWIZZLE_128B))
+        return fail(BO_ECUDA, "prefix fused-row: cuTensorMapEncodeTiled failed");
+    static bool attr = [] {
+        return cudaFuncSetAttribute(ps_fused_row_tma<T, INST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    static_cast<int>(C::kSmem)) == cudaSuccess;
+    }();
+    if (!attr) return fail(BO_ECUDA, "prefix fused-row: cannot set dynamic smem");
+    const long long ntiles = (p + INST - 1) / INST;
+    const int nchunks = static_cast<int>((n + fr::kElems - 1) / fr::kElems);
+    int per_sm = 1;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ps_fused_row_tma<T, INST>, INST, C::kSmem);
+    const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
+    static std::atomic<unsigned> next_slot{0};
+    const int slot = static_cast<int>(next_slot.fetch_add(1) % kWorkSlots);
+    ps_fused_row_tma<T, INST><<<static_cast<unsigned>(grid), INST, C::kSmem, st>>>(smap, dmap, ntiles, nchunks,
+                                                                                   slot);
+    return after_launch("ps_fused_row_tma");
 }
 
 template <typename T>
 static int launch_fused_row(const T *src, T *dst, int64_t n, int64_t p, cudaStream_t st) {
     if (fused_tma_ok(src, dst, n, p)) {
-        CUtensorMap smap, dmap;
-        if (!make_tmap_2d(&smap, src, p, n, fr::kInst, fr::kElems, CU_TENSOR_MAP_SWIZZLE_128B) ||
-            !make_tmap_2d(&dmap, dst, p, n, fr::kInst, fr::kElems, CU_TENSOR_MAP_SWIZZLE_128B))
-            return fail(BO_ECUDA, "prefix fused-row: cuTensorMapEncodeTiled failed");
-        static bool attr = [] {
-            return cudaFuncSetAttribute(ps_fused_row_tma<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        static_cast<int>(fr::kSmem)) == cudaSuccess;
-        }();
-        if (!attr) return fail(BO_ECUDA, "prefix fused-row: cannot set dynamic smem");
-        const long long ntiles = (p + fr::kInst - 1) / fr::kInst;
-        const int nchunks = static_cast<int>((n + fr::kElems - 1) / fr::kElems);
-        const long long grid = std::min<long long>(ntiles, 2LL * num_sms());
-        static std::atomic<unsigned> next_slot{0};
-        const int slot = static_cast<int>(next_slot.fetch_add(1) % kWorkSlots);
-        ps_fused_row_tma<T><<<static_cast<unsigned>(grid), fr::kInst, fr::kSmem, st>>>(smap, dmap, ntiles,
-                                                                                     nchunks, slot);
-        return after_launch("ps_fused_row_tma");
+        if (p < 2LL * 128 * num_sms()) return launch_fused_row_tma<T, 32>(src, dst, n, p, st);
+        return launch_fused_row_tma<T, 128>(src, dst, n, p, st);
     }
     const long long blocks = std::min<long long>((p + 127) / 128, 16LL * num_sms());
     ps_fused_row_smem<T><<<static_cast<unsigned>(blocks), 128, 0, st>>>(src, dst, n, p);
