@@ -58,8 +58,12 @@ WORKLOADS = {
                 desc="bulk optimal triangulation fp32 n=64, p=65536 (BASELINE configs[3])"),
     "tr2umm": dict(seed=4, algo="tri", n=64, p=65536, dtype="float32", layout=1, variant=16,
                    desc="the paper's column-wise UMM kernel on TR-2"),
+    "tr1col": dict(seed=3, algo="tri", n=16, p=65536, dtype="int32", layout=1, variant=0,
+                   desc="bulk optimal triangulation int32 n=16, p=65536, column-wise weights"),
+    "ps2naive_row": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=5,
+                         desc="the paper's row-wise kernel (thread per instance, uncoalesced)"),
 }
-EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr2", "ps2naive_col", "tr2umm"]
+EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr2", "ps2naive_col", "ps2naive_row", "tr2umm"]
 L2_BYTES = 126 * 2 ** 20
 
 
@@ -93,7 +97,7 @@ def load_peaks():
 
 
 def load_traffic():
-    path = os.path.join(ROOT, "profiles", "traffic.json")
+    path = os.path.join(ROOT, "profiles", "traffic.json")   # workload -> ncu DRAM bytes per launch
     try:
         with open(path) as f:
             return json.load(f)
@@ -178,11 +182,8 @@ class Ctx:
             dist.barrier(device_ids=[self.local])
 
     def max(self, x: float) -> float:
-        if not self.dist:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+        from paper_conf_ipps_tanitni14_b200 import shard
+        return shard.max_over_ranks(x)
 
 
 def timed(ctx, fn, steps, warmup, stream, flush=None):
@@ -229,7 +230,8 @@ def setup_workload(wl, rank):
     import paper_conf_ipps_tanitni14_b200 as bo
     n, p = wl["n"], wl["p"]
     dt = getattr(torch, wl["dtype"])
-    h0 = rank * p
+    from paper_conf_ipps_tanitni14_b200 import shard
+    h0, _ = shard.weak_range(p, rank)
     seed = wl["seed"]
     if wl["algo"] == "prefix":
         x = bo.generate_prefix(n, p, seed, dt, wl["layout"], "uniform", h0=h0)
@@ -428,7 +430,7 @@ def run_ours(args, ctx):
     bytes_launch = algo_bytes_per_instance(wl) * wl["p"]
     if wl["algo"] == "prefix":
         ach = bytes_launch / (per_launch_ms * 1e-3) / 1e9
-        tr = traffic.get(st["variant"], {}).get(name)
+        tr = traffic.get(name, {}).get("dram_bytes_per_launch")
         line["roofline"] = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                             "frac": ach / peaks["hbm_gbs"], "traffic": tr,
                             "peak_source": peak_src + " hbm_gbs (burst copy)",
@@ -438,17 +440,16 @@ def run_ours(args, ctx):
         ach = ops / (per_launch_ms * 1e-3) / 1e12
         pk = alu_peak_taddmin(peaks, wl["dtype"])
         line["roofline"] = {"bound": "alu", "achieved": ach, "peak": pk, "unit": "T add-min/s",
-                            "frac": ach / pk, "traffic": traffic.get(st["variant"], {}).get(name)}
+                            "frac": ach / pk, "traffic": traffic.get(name, {}).get("dram_bytes_per_launch")}
     line["clocks"] = sampler.summary()
     # checksum of each rank's shard, one NCCL all-gather (SURVEY §8 e), off the timed region
+    from paper_conf_ipps_tanitni14_b200 import shard
     cs = bo.checksum(st["out"], wl["layout"] if wl["algo"] == "prefix" else 0, h0=st["h0"])
-    if ctx.dist:
-        allcs = [torch.zeros_like(cs) for _ in range(ctx.world)]
-        dist.all_gather(allcs, cs)
-        cs_list = [int(c.cpu().numpy().view(np.uint64)[0]) for c in allcs]
-    else:
-        cs_list = [int(cs.cpu().numpy().view(np.uint64)[0])]
-    line["checksums"] = [hex(c) for c in cs_list]
+    cs_list = shard.gather_checksums(int(cs.cpu().numpy().view(np.uint64)[0]))
+    line["checksums"] = {"per_rank": [hex(c) for c in cs_list],
+                         "combined": hex(shard.combine_checksums(cs_list)),
+                         "note": "one NCCL all-gather after the timed region; inputs are generated per rank "
+                                 "from global instance ids, so nothing crosses NVLink on the data path"}
     if args.extras:
         ex = {}
         for e in EXTRAS:

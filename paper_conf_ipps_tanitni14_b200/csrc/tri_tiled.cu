@@ -138,11 +138,17 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long 
         // Only the weights Algorithm OPT reads (b >= a+2) are fetched.
         if (layout == BO_ROW_WISE && c_vec) {
             const T *ch = c + (live ? h : 0) * nn;
-            // warm L2 with this lane-group's NEXT instance while this one computes
-            if (li == 0 && h + inst_stride < p)
-                asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(c + (h + inst_stride) * nn),
-                             "r"(static_cast<unsigned>(nn * sizeof(T)))
-                             : "memory");
+            // warm L2 with the next instance this lane group will process: only the
+            // row segments Algorithm OPT reads (b >= a+2), one bulk prefetch per row
+            if (h + inst_stride < p) {
+                const T *cn = c + (h + inst_stride) * nn;
+                for (int a = li; a < n - 2; a += LPI) {
+                    const int m0 = (a + 2) >> 2;
+                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cn + static_cast<long long>(a) * n + 4 * m0),
+                                 "r"(static_cast<unsigned>((n - 4 * m0) * sizeof(T)))
+                                 : "memory");
+                }
+            }
             // lane li copies chunk m0(a)+li of row a; LPI=32 handles two rows per step
             for (int a0 = 0; a0 < n - 2; a0 += LPI / 16) {
                 const int a = a0 + (li >> 4);

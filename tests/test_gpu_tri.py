@@ -21,13 +21,13 @@ def _variants(n):
     v = [bo.AUTO, bo.TRI_UMM_GLOBAL, bo.TRI_SMEM_WARP]
     if n <= 18:
         v.append(bo.TRI_THREAD_REG)
-    if bo.triangulation_variant(n, 1, bo.F32, bo.ROW_WISE, bo.AUTO) == bo.TRI_TILED or 5 <= n <= 64:
-        v.append(bo.TRI_TILED)
+    if 5 <= n <= 64:
+        v += [bo.TRI_TILED, bo.TRI_TILED_HALF]
     return v
 
 
 def _supported(n, variant):
-    if variant == bo.TRI_TILED:
+    if variant in (bo.TRI_TILED, bo.TRI_TILED_HALF):
         try:
             bo.triangulation(torch.zeros((1, n, n), device=DEV), bo.ROW_WISE, bo.TRI_TILED)
         except bo.BulkError as e:
@@ -98,7 +98,7 @@ def test_tr2_full_config(layout):
     assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32))
 
 
-@pytest.mark.parametrize("variant", [bo.TRI_SMEM_WARP, bo.TRI_TILED, bo.TRI_UMM_GLOBAL])
+@pytest.mark.parametrize("variant", [bo.TRI_SMEM_WARP, bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_UMM_GLOBAL])
 def test_tr2_variants_agree_full_size(variant):
     n, p = 64, 65536
     c = bo.generate_tri(n, p, 4, torch.float32, bo.ROW_WISE)
