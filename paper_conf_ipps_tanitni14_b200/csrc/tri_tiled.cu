@@ -10,21 +10,27 @@
 // the same sums in the same association, and out = X[0][n-1] = M[1,n-1].
 // c[a][b] and X[a][b] share coordinates, so c is preloaded into the table.
 //
-// Shared-memory table Z (NP = 4*ceil(n/4) rows, row stride 68 elements):
-//   Z[a][b] = X[a][b] for b > a (initially c[a][b]),  Z[b][a] = X[a][b].
+// Shared-memory table: the UPPER triangle only, stored by 4-wide column
+// chunks ("chunk-columns"): chunk-column m holds rows 0..4m+3 (+1 pad row) of
+// columns 4m..4m+3, so element X[a][b] lives at chunk colbase(b/4) + a, word
+// b%4, with colbase(m) = 2m^2 + 3m (heights 4m+5 are odd, which spreads the
+// quarter-warp's chunks over all 8 bank groups).  8.75 KB per instance at
+// n = 64 instead of a 16 KB square, so twice as many instances per SM.
+// Before a cell is computed it holds c[a][b] (preloaded with cp.async).
 // For a tile (I,J), I < J (rows 4I..4I+3, cols 4J..4J+3) the k range splits
-//   k in [4I+4, 4J-1]  -> min-plus "dot product" of row-blocks I and J of Z
-//                         over aligned 4-wide column chunks m = I+1..J-1:
-//                         S[u][v] = min_m min_w Z[4I+u][4m+w] + Z[4J+v][4m+w]
+//   k in [4I+4, 4J-1]  -> dense min-plus product over chunk-columns m = I+1..J-1:
+//                         A_u = X[4I+u][4m..4m+3]   (chunk-column m, rows 4I+u)
+//                         B_w = X[4m+w][4J..4J+3]   (chunk-column J, rows 4m+w)
+//                         S[u][v] = min_w A_u[w] + B_w[v]
 //   k in (a, 4I+3]     -> P1: diagonal tile (I,I) x rows of this tile below
 //   k in [4J, b)       -> P3: columns of this tile to the left x tile (J,J)
-// One chunk = 8 LDS.128 + 64 add-mins; consecutive k sit in adjacent
-// registers, so fp32 runs as FADD2 + FMNMX3 (one instruction per add-min)
-// and int32 as VIADDMNMX.  P1/P3 are a 4x4 triangular solve in registers.
-// Tiles of one tile-diagonal D = J-I are independent; long dense ranges are
-// split over s lanes and min-reduced with xor shuffles.  Row stride 68 puts
-// chunk m of row r in bank group (r + m) mod 8 and keeps a tile's four rows
-// at immediate offsets.
+// One chunk = 8 LDS.128 (each row read at an immediate offset) + 64
+// add-mins; fp32 pairs two v's in one FADD2 with the A value broadcast
+// (FADD2 Rd, Ra.F32, Rb.F32x2) and folds two k's per FMNMX3 -- one
+// instruction per add-min; int32 is one VIADDMNMX per add-min.  P1/P3 are
+// a 4x4 triangular solve in registers ("fix-up").  Tiles of one
+// tile-diagonal D = J-I are independent; long dense ranges are split over s
+// lanes and min-reduced with xor shuffles.
 #include "common.cuh"
 
 #include <climits>
@@ -65,7 +71,10 @@ template <typename T> struct V4;
 template <> struct V4<float> { using type = float4; };
 template <> struct V4<int32_t> { using type = int4; };
 
-constexpr int kRS = 68;   // row stride (elements)
+// chunk-column m starts at chunk colbase(m); element (a, b) at word xoff(a, b)
+__host__ __device__ __forceinline__ constexpr int colbase(int m) { return 2 * m * m + 3 * m; }
+__device__ __forceinline__ int xc(int a, int m) { return 4 * (colbase(m) + a); }   // chunk (row a, col-chunk m)
+__device__ __forceinline__ int xoff(int a, int b) { return xc(a, b >> 2) + (b & 3); }
 
 template <typename T>
 __device__ __forceinline__ typename V4<T>::type ld4(const T *p) {
@@ -86,18 +95,32 @@ __device__ __forceinline__ void cp_async16(void *dst, const void *src, bool pred
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
-// 16 partial tiles: consecutive k pairs (w, w+1) come from one 128-bit load
-template <typename T>
-__device__ __forceinline__ void minplus_chunk(T (&acc)[4][4], const typename V4<T>::type (&A)[4],
-                                              const typename V4<T>::type (&B)[4]) {
-    using T2 = typename V2<T>::type;
+// S[u][v] = min(S[u][v], min_w A[u].w + B[w].v) for one 4-wide k chunk
+__device__ __forceinline__ float comp(const float4 &v, int i) { return i == 0 ? v.x : i == 1 ? v.y : i == 2 ? v.z : v.w; }
+__device__ __forceinline__ int comp(const int4 &v, int i) { return i == 0 ? v.x : i == 1 ? v.y : i == 2 ? v.z : v.w; }
+
+__device__ __forceinline__ void minplus_chunk(float (&acc)[4][4], const float4 (&A)[4], const float4 (&B)[4]) {
 #pragma unroll
     for (int u = 0; u < 4; ++u)
 #pragma unroll
-        for (int v = 0; v < 4; ++v) {
-            const T x = Ops<T>::addmin2(T2{A[u].x, A[u].y}, T2{B[v].x, B[v].y}, acc[u][v]);
-            acc[u][v] = Ops<T>::addmin2(T2{A[u].z, A[u].w}, T2{B[v].z, B[v].w}, x);
+        for (int w = 0; w < 4; w += 2) {
+            const float a0 = comp(A[u], w), a1 = comp(A[u], w + 1);
+#pragma unroll
+            for (int v = 0; v < 4; v += 2) {
+                const float2 s0 = __fadd2_rn(make_float2(a0, a0), make_float2(comp(B[w], v), comp(B[w], v + 1)));
+                const float2 s1 = __fadd2_rn(make_float2(a1, a1), make_float2(comp(B[w + 1], v), comp(B[w + 1], v + 1)));
+                acc[u][v] = fminf(fminf(acc[u][v], s0.x), s1.x);
+                acc[u][v + 1] = fminf(fminf(acc[u][v + 1], s0.y), s1.y);
+            }
         }
+}
+__device__ __forceinline__ void minplus_chunk(int32_t (&acc)[4][4], const int4 (&A)[4], const int4 (&B)[4]) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int w = 0; w < 4; ++w)
+#pragma unroll
+            for (int v = 0; v < 4; ++v) acc[u][v] = __viaddmin_s32(comp(A[u], w), comp(B[w], v), acc[u][v]);
 }
 }  // namespace tt
 
@@ -114,17 +137,17 @@ __global__ void __launch_bounds__(128, 1)
 tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long p, int layout, int NT, int c_vec) {
     using Op = tt::Ops<T>;
     using T4 = typename tt::V4<T>::type;
-    using tt::kRS;
+    using tt::xc;
     constexpr int IPW = 32 / LPI;                       // instances per warp
     extern __shared__ uint8_t smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int slot = lane / LPI, li = lane % LPI;       // instance slot in warp, lane in instance
-    const int NP = 4 * NT;
+    const int words = 4 * tt::colbase(NT);            // per-instance table size
     const int warps_per_cta = blockDim.x >> 5;
-    T *Z = reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warp * IPW + slot) * NP * kRS;
+    T *Z = reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warp * IPW + slot) * words;
 
-    // zero the table once: padding rows / columns then stay finite forever
-    for (int i = li; i < NP * kRS; i += LPI) Z[i] = T(0);
+    // zero the table once: padding cells then stay finite forever
+    for (int i = li; i < words; i += LPI) Z[i] = T(0);
     __syncwarp();
 
     const long long inst_stride = static_cast<long long>(gridDim.x) * warps_per_cta * IPW;
@@ -138,29 +161,27 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long 
         // Only the weights Algorithm OPT reads (b >= a+2) are fetched.
         if (layout == BO_ROW_WISE && c_vec) {
             const T *ch = c + (live ? h : 0) * nn;
-            // warm L2 with the next instance this lane group will process: only the
-            // row segments Algorithm OPT reads (b >= a+2), one bulk prefetch per row
-            if (h + inst_stride < p) {
-                const T *cn = c + (h + inst_stride) * nn;
-                for (int a = li; a < n - 2; a += LPI) {
-                    const int m0 = (a + 2) >> 2;
-                    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(cn + static_cast<long long>(a) * n + 4 * m0),
-                                 "r"(static_cast<unsigned>((n - 4 * m0) * sizeof(T)))
-                                 : "memory");
+            // Row block g = rows 4g..4g+3: lane li copies chunk-column m = g + li of
+            // all four rows (four consecutive 16-byte chunks in the table).  Rows
+            // 4g+2, 4g+3 also bring their diagonal chunk g, which D = 0 overwrites.
+            // LPI = 32: lanes 16..31 take the odd row blocks.
+            if (live) {
+                for (int g = li >> 4; g < NT; g += LPI / 16) {
+                    const int m = g + (li & 15);
+                    if (m <= last_chunk) {
+                        T *dst = Z + xc(4 * g, m);
+                        const T *src = ch + static_cast<long long>(4 * g) * n + 4 * m;
+#pragma unroll
+                        for (int r = 0; r < 4; ++r)
+                            tt::cp_async16(dst + 4 * r, src + static_cast<long long>(r) * n, 4 * g + r < n - 2);
+                    }
                 }
-            }
-            // lane li copies chunk m0(a)+li of row a; LPI=32 handles two rows per step
-            for (int a0 = 0; a0 < n - 2; a0 += LPI / 16) {
-                const int a = a0 + (li >> 4);
-                const int m = ((a + 2) >> 2) + (li & 15);
-                tt::cp_async16(Z + a * kRS + 4 * m, ch + static_cast<long long>(a) * n + 4 * m,
-                           live && a < n - 2 && m <= last_chunk);
             }
             tt::cp_async_wait_all();
         } else if (live) {
             for (int a = 0; a < n - 2; ++a)
                 for (int b = a + 2 + li; b < n; b += LPI)
-                    Z[a * kRS + b] = __ldg(c + (layout == BO_ROW_WISE ? h * nn + static_cast<long long>(a) * n + b
+                    Z[tt::xoff(a, b)] = __ldg(c + (layout == BO_ROW_WISE ? h * nn + static_cast<long long>(a) * n + b
                                                                       : (static_cast<long long>(a) * n + b) * p + h));
         }
         __syncwarp();
@@ -168,17 +189,17 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long 
         // ------------------------------------------------ 2. D = 0 (diagonal tiles)
         if (li < NT) {
             const int I = li;
-            T *r0 = Z + (4 * I) * kRS + 4 * I;
-            const T4 c0 = tt::ld4(r0), c1 = tt::ld4(r0 + kRS);
+            T *r0 = Z + xc(4 * I, I);                    // rows 4I.. of chunk-column I
+            const T4 c0 = tt::ld4(r0), c1 = tt::ld4(r0 + 4);
             const T z = T(0);
             // X[a][a+1] = 0; X[0][2], X[1][3] have the single k with two zero terms
             const T t02 = Op::add(Op::add(z, z), c0.z);
             const T t13 = Op::add(Op::add(z, z), c1.w);
             const T t03 = Op::add(Op::min(Op::add(z, t13), Op::add(t02, z)), c0.w);
-            tt::st4(r0, z, z, t02, t03);
-            tt::st4(r0 + kRS, z, z, z, t13);
-            tt::st4(r0 + 2 * kRS, t02, z, z, z);
-            tt::st4(r0 + 3 * kRS, t03, t13, z, z);
+            tt::st4(r0, z, z, t02, t03);                 // below-diagonal words are unused
+            tt::st4(r0 + 4, z, z, z, t13);
+            tt::st4(r0 + 8, z, z, z, z);
+            tt::st4(r0 + 12, z, z, z, z);
         }
         __syncwarp();
 
@@ -196,33 +217,34 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long 
                 for (int v = 0; v < 4; ++v) acc[u][v] = Op::inf();
             if (act) {
                 int m = I + 1 + q;
-                const T *pa = Z + (4 * I) * kRS + 4 * m;
-                const T *pb = Z + (4 * J) * kRS + 4 * m;
+                const T *pa = Z + xc(4 * I, m);                 // A rows 4I+u: pa + 4u
+                const T *pb = Z + xc(4 * m, J);                 // B rows 4m+w: pb + 4w
+                const int db = 16 * s;                          // B: next chunk = 4s rows further down
                 if (m < J) {
                     // software-pipelined ping-pong: load chunk m+s while computing chunk m
                     T4 A0[4], B0[4], A1[4], B1[4];
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + u * kRS), B0[u] = tt::ld4(pb + u * kRS);
+                    for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + 4 * u), B0[u] = tt::ld4(pb + 4 * u);
                     while (true) {
+                        pa += 4 * (4 * m * s + 2 * s * s + 3 * s);   // colbase(m+s) - colbase(m) chunks
+                        pb += db;
                         m += s;
-                        pa += 4 * s;
-                        pb += 4 * s;
                         bool more = m < J;
                         if (more) {
 #pragma unroll
-                            for (int u = 0; u < 4; ++u) A1[u] = tt::ld4(pa + u * kRS), B1[u] = tt::ld4(pb + u * kRS);
+                            for (int u = 0; u < 4; ++u) A1[u] = tt::ld4(pa + 4 * u), B1[u] = tt::ld4(pb + 4 * u);
                         }
-                        tt::minplus_chunk<T>(acc, A0, B0);
+                        tt::minplus_chunk(acc, A0, B0);
                         if (!more) break;
+                        pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
+                        pb += db;
                         m += s;
-                        pa += 4 * s;
-                        pb += 4 * s;
                         more = m < J;
                         if (more) {
 #pragma unroll
-                            for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + u * kRS), B0[u] = tt::ld4(pb + u * kRS);
+                            for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + 4 * u), B0[u] = tt::ld4(pb + 4 * u);
                         }
-                        tt::minplus_chunk<T>(acc, A1, B1);
+                        tt::minplus_chunk(acc, A1, B1);
                         if (!more) break;
                     }
                 }
@@ -236,13 +258,13 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long 
             if (act && q == 0) {
                 // A[u][w] = X[4I+u][4I+w] (w > u), Bd[w][v] = X[4J+w][4J+v] (v > w),
                 // C[u][v] = c[4I+u][4J+v] (still in the tile's own upper cells)
-                T *ta = Z + (4 * I) * kRS + 4 * I;
-                T *tb = Z + (4 * J) * kRS + 4 * J;
-                T *tc = Z + (4 * I) * kRS + 4 * J;
+                T *ta = Z + xc(4 * I, I);
+                T *tb = Z + xc(4 * J, J);
+                T *tc = Z + xc(4 * I, J);
                 T A[4][4], Bd[4][4], C[4][4];
 #pragma unroll
                 for (int r = 0; r < 4; ++r) {
-                    const T4 x = tt::ld4(ta + r * kRS), y = tt::ld4(tb + r * kRS), w = tt::ld4(tc + r * kRS);
+                    const T4 x = tt::ld4(ta + 4 * r), y = tt::ld4(tb + 4 * r), w = tt::ld4(tc + 4 * r);
                     A[r][0] = x.x; A[r][1] = x.y; A[r][2] = x.z; A[r][3] = x.w;
                     Bd[r][0] = y.x; Bd[r][1] = y.y; Bd[r][2] = y.z; Bd[r][3] = y.w;
                     C[r][0] = w.x; C[r][1] = w.y; C[r][2] = w.z; C[r][3] = w.w;
@@ -262,14 +284,11 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long 
                         if (u == 3 && v == 0 && D == 1) t[u][v] = T(0);
                     }
 #pragma unroll
-                for (int u = 0; u < 4; ++u) tt::st4(tc + u * kRS, t[u][0], t[u][1], t[u][2], t[u][3]);
-                T *tl = Z + (4 * J) * kRS + 4 * I;      // transpose into the lower part
-#pragma unroll
-                for (int v = 0; v < 4; ++v) tt::st4(tl + v * kRS, t[0][v], t[1][v], t[2][v], t[3][v]);
+                for (int u = 0; u < 4; ++u) tt::st4(tc + 4 * u, t[u][0], t[u][1], t[u][2], t[u][3]);
             }
             __syncwarp();
         }
-        if (live && li == 0) out[h] = Z[n - 1];          // X[0][n-1] = Algorithm OPT's M[1,n-1]
+        if (live && li == 0) out[h] = Z[tt::xoff(0, n - 1)];   // X[0][n-1] = Algorithm OPT's M[1,n-1]
         __syncwarp();
     }
 }
@@ -279,7 +298,7 @@ int tiled_supported(int64_t n) { return n >= 5 && n <= 64; }
 template <typename T, int LPI>
 static int launch_tiled_t(const void *c, void *out, int64_t n, int64_t p, int layout, cudaStream_t st) {
     const int NT = static_cast<int>((n + 3) / 4);
-    const size_t per_inst = static_cast<size_t>(4 * NT) * tt::kRS * sizeof(T);
+    const size_t per_inst = static_cast<size_t>(4 * tt::colbase(NT)) * sizeof(T);
     constexpr int IPW = 32 / LPI;
     // warps per CTA: the W in 1..4 that keeps the most warps resident per SM
     // (shared memory is the limit: 227 KB, 1 KB reserved per CTA)
