@@ -61,6 +61,14 @@ def lib():
         L.oracle_bulk_prefix.restype = i32
         L.oracle_bulk_opt.argtypes = [vp, vp, i64, i64, i32, i32, i64, i64, i32]
         L.oracle_bulk_opt.restype = i32
+        L.oracle_opt_chords_i32.argtypes = [vp, i64, vp]
+        L.oracle_opt_chords_i32.restype = ctypes.c_int32
+        L.oracle_opt_chords_f32.argtypes = [vp, i64, vp]
+        L.oracle_opt_chords_f32.restype = ctypes.c_float
+        L.oracle_brute_opt_set_f64.argtypes = [vp, i64, vp]
+        L.oracle_brute_opt_set_f64.restype = ctypes.c_double
+        L.oracle_bulk_opt_chords.argtypes = [vp, vp, vp, i64, i64, i32, i32, i64, i64]
+        L.oracle_bulk_opt_chords.restype = i32
         _lib = L
     return _lib
 
@@ -166,6 +174,44 @@ def bulk_opt(c: np.ndarray, layout: int, nthreads: int = 1,
     rc = lib().oracle_bulk_opt(_ptr(c), _ptr(out), n, p, _DT[_dtname(c)], layout, h0, h1, nthreads)
     assert rc == 0
     return out
+
+
+def opt_chords(c: np.ndarray):
+    """Algorithm OPT with argmin bookkeeping (first minimising k as the
+    strict '<' of P:196 keeps it) and the pre-order chord read-out.
+    Returns (value, chords [n-3, 2] int16 of vertex pairs (a, b), a < b)."""
+    c = np.ascontiguousarray(c)
+    n = c.shape[0]
+    ch = np.zeros((max(n - 3, 0), 2), dtype=np.int16)
+    if _dtname(c) == "int32":
+        v = lib().oracle_opt_chords_i32(_ptr(c), n, _ptr(ch))
+    else:
+        v = lib().oracle_opt_chords_f32(_ptr(c), n, _ptr(ch))
+    return c.dtype.type(v), ch
+
+
+def brute_opt_set(c: np.ndarray):
+    """Brute-force optimum + the chord set of the first optimal triangulation
+    found in lexicographic chord order; returns (value float64, chords [n-3, 2])."""
+    w = np.ascontiguousarray(c, dtype=np.float64)
+    n = w.shape[0]
+    ch = np.zeros((max(n - 3, 0), 2), dtype=np.int16)
+    v = lib().oracle_brute_opt_set_f64(_ptr(w), n, _ptr(ch))
+    return v, ch
+
+
+def bulk_opt_chords(c: np.ndarray, layout: int):
+    """Parallel Algorithm OPT with chords for every instance: (out[p], chords[p, n-3, 2])."""
+    c = np.ascontiguousarray(c)
+    if layout == ROW_WISE:
+        p, n, _ = c.shape
+    else:
+        n, _, p = c.shape
+    out = np.zeros(p, dtype=c.dtype)
+    ch = np.zeros((p, max(n - 3, 0), 2), dtype=np.int16)
+    rc = lib().oracle_bulk_opt_chords(_ptr(c), _ptr(out), _ptr(ch), n, p, _DT[_dtname(c)], layout, 0, p)
+    assert rc == 0
+    return out, ch
 
 
 # ----------------------------------------------------------------- transpose

@@ -163,3 +163,70 @@ def test_bulk_row_and_column_arrangements(dt):
     assert np.array_equal(r.view(np.uint32), c.view(np.uint32))
     for h in range(p):
         assert r[h] == oracle.opt(row[h])
+
+
+# ------------------------------------------------- NEXT-1: the triangulation itself
+def _check_triangulation(chords, n):
+    chords = [tuple(int(x) for x in ch) for ch in chords]
+    assert len(chords) == n - 3 and len(set(chords)) == n - 3
+    for a, b in chords:
+        assert 0 <= a < b < n and b - a >= 2 and (a, b) != (0, n - 1)
+    for i, (a, b) in enumerate(chords):
+        for x, y in chords[i + 1:]:
+            assert not ((a < x < b < y) or (x < a < y < b)), "crossing chords"
+    return chords
+
+
+@pytest.mark.parametrize("n", [3, 4, 5, 6, 9, 16, 40])
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+def test_chords_form_a_triangulation_of_the_optimal_weight(n, dt):
+    for h in range(5):
+        c = bulkgen.tri_instances(n, [h], seed=300 + n, dtype=dt)[0]
+        v, ch = oracle.opt_chords(c)
+        assert v == oracle.opt(c)
+        chords = _check_triangulation(ch, n)
+        total = sum(float(c[a, b]) for a, b in chords) + float(c[0, n - 1])
+        if dt == "int32":
+            assert int(total) == int(v)
+        else:
+            assert abs(total - float(v)) <= (n + 1) * 2.0 ** -24 * max(float(v), 1e-30)
+
+
+@pytest.mark.parametrize("n", range(5, 11))
+def test_chords_equal_brute_force_set_when_optimum_unique(n):
+    for h in range(4):
+        c = bulkgen.tri_instances(n, [h], seed=400 + n, dtype="int32")[0]
+        bv, bset = oracle.brute_opt_set(c)
+        v, ch = oracle.opt_chords(c)
+        assert int(bv) == int(v)
+        # weights are 20-bit random integers: the optimum is unique w.h.p.; check it is
+        assert sorted(map(tuple, bset.tolist())) == sorted(map(tuple, ch.tolist()))
+
+
+def test_chords_of_hand_worked_pentagon():
+    c, (value, _) = _parse_worked("pentagon_worked.txt")
+    v, ch = oracle.opt_chords(c)
+    assert int(v) == value
+    assert sorted(map(tuple, ch.tolist())) == [(0, 3), (1, 3)]       # fan at v3 (golden)
+
+
+def test_chords_tie_break_is_first_k():
+    # n = 4, equal diagonals: the strict '<' keeps k = i -> right part (1,3)
+    c = np.zeros((4, 4), dtype=np.int32)
+    c[0, 2] = c[1, 3] = 5
+    v, ch = oracle.opt_chords(c)
+    assert int(v) == 5 and ch.tolist() == [[1, 3]]
+    c[1, 3] = 6
+    assert oracle.opt_chords(c)[1].tolist() == [[0, 2]]
+
+
+def test_bulk_chords_layouts_agree():
+    n, p = 12, 9
+    row = bulkgen.tri_input(n, p, seed=5, dtype="float32", layout=bulkgen.ROW_WISE)
+    col = bulkgen.tri_input(n, p, seed=5, dtype="float32", layout=bulkgen.COLUMN_WISE)
+    a, ca = oracle.bulk_opt_chords(row, oracle.ROW_WISE)
+    b, cb = oracle.bulk_opt_chords(col, oracle.COLUMN_WISE)
+    assert np.array_equal(a, b) and np.array_equal(ca, cb)
+    for h in range(p):
+        v, ch = oracle.opt_chords(row[h])
+        assert v == a[h] and np.array_equal(ch, ca[h])
