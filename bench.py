@@ -60,10 +60,12 @@ WORKLOADS = {
                    desc="the paper's column-wise UMM kernel on TR-2"),
     "tr1col": dict(seed=3, algo="tri", n=16, p=65536, dtype="int32", layout=1, variant=0,
                    desc="bulk optimal triangulation int32 n=16, p=65536, column-wise weights"),
+    "tr2chords": dict(seed=4, algo="tri", n=64, p=65536, dtype="float32", layout=0, variant="chords",
+                      desc="NEXT-1: TR-2 values plus the chords of each optimal triangulation"),
     "ps2naive_row": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=5,
                          desc="the paper's row-wise kernel (thread per instance, uncoalesced)"),
 }
-EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr2", "ps2naive_col", "ps2naive_row", "tr2umm"]
+EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr2", "tr2chords", "ps2naive_col", "ps2naive_row", "tr2umm"]
 L2_BYTES = 126 * 2 ** 20
 
 
@@ -250,6 +252,10 @@ def setup_workload(wl, rank):
         x = bo.generate_tri(n, p, seed, dt, wl["layout"], h0=h0)
         out = torch.empty(p, dtype=dt, device="cuda")
         dcode = bo.F32 if wl["dtype"] == "float32" else bo.I32
+        if wl["variant"] == "chords":
+            def fn():
+                bo.triangulation_chords(x, wl["layout"])
+            return dict(x=x, out=out, fn=fn, seed=seed, h0=h0, variant="tiled_half+chords")
         need = bo.triangulation_workspace(n, p, dcode, wl["layout"], wl["variant"])
         ws = torch.empty(need, dtype=torch.uint8, device="cuda") if need else None
 

@@ -120,6 +120,20 @@ int bulk_triangulation(const void *c, void *out, int64_t n, int64_t p, int dtype
 size_t bulk_triangulation_workspace(int64_t n, int64_t p, int dtype, int layout, int variant);
 
 /* ------------------------------------------------------------------------- */
+/* The optimal triangulation itself (NEXT-1; "a few extra bookkeeping steps", */
+/* P:157).  out[h] as bulk_triangulation; chords[h] = the n-3 chords of the   */
+/* triangulation Algorithm OPT selects when its strict "<" keeps the */
+/* FIRST minimising k.  Order: sub-polygons are split depth first from the    */
+/* root side (v0, v_{n-1}), left part first; each split of (a, b) at k emits  */
+/* (a, k) then (k, b) if that part has >= 3 vertices.                          */
+/*   chords : device int16, [p][n-3][2] vertex pairs (a, b), a < b.           */
+/*   3 <= n <= 64 (BO_EUNSUPPORTED above), same c layouts and weight          */
+/*   preconditions as bulk_triangulation.                                     */
+/* ------------------------------------------------------------------------- */
+int bulk_triangulation_chords(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int dtype,
+                              int layout, void *stream);
+
+/* ------------------------------------------------------------------------- */
 /* Layout transpose (row-wise <-> column-wise arrangement):        */
 /*   dst[c*rows + r] = src[r*cols + c],  0 <= r < rows, 0 <= c < cols.        */
 /* Row-wise [p][n] -> column-wise [n][p] is (rows=p, cols=n); the reverse is  */

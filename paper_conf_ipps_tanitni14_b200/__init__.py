@@ -58,6 +58,7 @@ def lib() -> ctypes.CDLL:
             "bulk_triangulation": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_triangulation_workspace": ([i64, i64, i32, i32, i32], sz),
             "bulk_transpose": ([vp, vp, i64, i64, sz, vp], i32),
+            "bulk_triangulation_chords": ([vp, vp, vp, i64, i64, i32, i32, vp], i32),
             "bulk_prefix_sums_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_triangulation_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_generate_prefix": ([vp, i64, i64, i64, u64, i32, i32, i32, vp], i32),
@@ -194,6 +195,19 @@ def triangulation(c: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, 
     _check(lib().bulk_triangulation(c.data_ptr(), out.data_ptr(), n, p, dt, layout, variant, wptr, wbytes,
                                     _stream(stream)))
     return out
+
+
+def triangulation_chords(c: torch.Tensor, layout: int = ROW_WISE, stream=None):
+    """Values and the chords of an optimal triangulation (NEXT-1):
+    returns (out [p], chords [p, n-3, 2] int16 vertex pairs)."""
+    _need_cuda(c)
+    n, p = _tri_shape(c, layout)
+    dt = _dtype_code(c)
+    out = torch.empty(p, dtype=c.dtype, device=c.device)
+    chords = torch.empty((p, max(n - 3, 0), 2), dtype=torch.int16, device=c.device)
+    _check(lib().bulk_triangulation_chords(c.data_ptr(), out.data_ptr(), chords.data_ptr() if chords.numel() else None,
+                                           n, p, dt, layout, _stream(stream)))
+    return out, chords
 
 
 def triangulation_host(c_host: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO,

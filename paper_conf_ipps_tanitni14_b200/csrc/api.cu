@@ -59,6 +59,8 @@ int resolve_prefix_variant(int64_t n, int64_t p, int layout, int variant, const 
 int tri_dispatch(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int variant, void *ws,
                  cudaStream_t st);
 int resolve_tri_variant(int64_t n, int64_t p, int dtype, int layout, int variant);
+int launch_tri_chords(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int dtype, int layout,
+                      cudaStream_t st);
 size_t tri_workspace(int64_t n, int64_t p, int variant);
 int launch_gen_prefix(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
 int launch_gen_tri(void *, int64_t, int64_t, int64_t, uint64_t, int, int, cudaStream_t);
@@ -205,6 +207,17 @@ int bulk_triangulation(const void *c, void *out, int64_t n, int64_t p, int dtype
     if (need > 0 && (!workspace || workspace_bytes < need))
         return fail(BO_EINVAL, "triangulation: workspace too small (need " + std::to_string(need) + " bytes)");
     return tri_dispatch(c, out, n, p, dtype, layout, v, workspace, static_cast<cudaStream_t>(stream));
+}
+
+int bulk_triangulation_chords(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int dtype,
+                              int layout, void *stream) {
+    t_err.clear();
+    int rc = check_tri_args(c, out, n, p, dtype, layout, BO_AUTO);
+    if (rc) return rc;
+    if (n > 64) return fail(BO_EUNSUPPORTED, "triangulation chords: n <= 64 (the table must fit in shared memory)");
+    if (p == 0) return BO_OK;
+    if (n > 3 && !chords) return fail(BO_EINVAL, "triangulation chords: NULL chords pointer");
+    return launch_tri_chords(c, out, chords, n, p, dtype, layout, static_cast<cudaStream_t>(stream));
 }
 
 int bulk_transpose(const void *src, void *dst, int64_t rows, int64_t cols, size_t elem_bytes, void *stream) {

@@ -132,9 +132,13 @@ __device__ __forceinline__ int split_log2(int t, int D, int lpi) {
     return ls;
 }
 
-template <typename T, int LPI>
+// Extra shared words per instance for the chord walk (stack of intervals).
+__host__ __device__ constexpr int chord_stack_words(int NT) { return 8 * NT + 4; }
+
+template <typename T, int LPI, bool CHORDS>
 __global__ void __launch_bounds__(128, 1)
-tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long p, int layout, int NT, int c_vec) {
+tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restrict__ chords, int n, long long p,
+                 int layout, int NT, int c_vec) {
     using Op = tt::Ops<T>;
     using T4 = typename tt::V4<T>::type;
     using tt::xc;
@@ -145,6 +149,8 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long 
     const int words = 4 * tt::colbase(NT);            // per-instance table size
     const int warps_per_cta = blockDim.x >> 5;
     T *Z = reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warp * IPW + slot) * words;
+    int *stk = reinterpret_cast<int *>(reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warps_per_cta) * IPW * words) +
+               static_cast<size_t>(warp * IPW + slot) * chord_stack_words(NT);
 
     // zero the table once: padding cells then stay finite forever
     for (int i = li; i < words; i += LPI) Z[i] = T(0);
@@ -289,16 +295,60 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int n, long long 
             __syncwarp();
         }
         if (live && li == 0) out[h] = Z[tt::xoff(0, n - 1)];   // X[0][n-1] = Algorithm OPT's M[1,n-1]
+        if constexpr (CHORDS) {
+            // NEXT-1: read the optimal triangulation off the finished table.
+            // Visit sub-polygons (a, b) depth first, left part first; the split of
+            // (a, b) is the smallest k with X[a][k] + X[k][b] equal to the min (the
+            // k Algorithm OPT's strict '<' keeps) -- recomputed here exactly,
+            // with the same fp32 adds.  Each split emits (a, k) then (k, b) when
+            // that part has >= 3 vertices.  Every instance has n-2 splits, so all
+            // lanes of the warp run the same number of iterations.
+            int sp = 2, t = 0;
+            if (li == 0) stk[0] = 0, stk[1] = n - 1;
+            __syncwarp();
+            int16_t *oc = chords + (live ? h : 0) * 2LL * (n - 3);
+            for (int it = 0; it < n - 2; ++it) {
+                sp -= 2;
+                const int a = stk[sp], b = stk[sp + 1];
+                T best = Op::inf();
+                int kb = n;
+                for (int k = a + 1 + li; k < b; k += LPI) {
+                    const T r = Op::add(Z[tt::xoff(a, k)], Z[tt::xoff(k, b)]);
+                    if (r < best) best = r, kb = k;
+                }
+#pragma unroll
+                for (int off = 1; off < LPI; off <<= 1) {
+                    const T ob = __shfl_xor_sync(0xffffffffu, best, off);
+                    const int ok = __shfl_xor_sync(0xffffffffu, kb, off);
+                    if (ob < best || (ob == best && ok < kb)) best = ob, kb = ok;
+                }
+                const int k = kb;
+                const bool left = k - a >= 2, right = b - k >= 2;
+                __syncwarp();
+                if (li == 0) {
+                    if (right) stk[sp] = k, stk[sp + 1] = b;
+                    if (left) stk[sp + 2 * right] = a, stk[sp + 2 * right + 1] = k;
+                    if (live) {
+                        if (left) oc[2 * t] = static_cast<int16_t>(a), oc[2 * t + 1] = static_cast<int16_t>(k);
+                        if (right) oc[2 * (t + left)] = static_cast<int16_t>(k), oc[2 * (t + left) + 1] = static_cast<int16_t>(b);
+                    }
+                }
+                sp += 2 * (left + right);
+                t += left + right;
+                __syncwarp();
+            }
+        }
         __syncwarp();
     }
 }
 
-int tiled_supported(int64_t n) { return n >= 5 && n <= 64; }
+int tiled_supported(int64_t n) { return n >= 3 && n <= 64; }
 
-template <typename T, int LPI>
-static int launch_tiled_t(const void *c, void *out, int64_t n, int64_t p, int layout, cudaStream_t st) {
+template <typename T, int LPI, bool CHORDS>
+static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int layout,
+                          cudaStream_t st) {
     const int NT = static_cast<int>((n + 3) / 4);
-    const size_t per_inst = static_cast<size_t>(4 * tt::colbase(NT)) * sizeof(T);
+    const size_t per_inst = static_cast<size_t>(4 * tt::colbase(NT) + (CHORDS ? chord_stack_words(NT) : 0)) * sizeof(T);
     constexpr int IPW = 32 / LPI;
     // warps per CTA: the W in 1..4 that keeps the most warps resident per SM
     // (shared memory is the limit: 227 KB, 1 KB reserved per CTA)
@@ -310,19 +360,19 @@ static int launch_tiled_t(const void *c, void *out, int64_t n, int64_t p, int la
     }
     const size_t smem = W * IPW * per_inst;
     static bool attr = [] {
-        return cudaFuncSetAttribute(tri_tiled_kernel<T, LPI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        return cudaFuncSetAttribute(tri_tiled_kernel<T, LPI, CHORDS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     227 * 1024) == cudaSuccess;
     }();
     if (!attr) return fail(BO_ECUDA, "tiled: cannot set dynamic smem");
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_tiled_kernel<T, LPI>, W * 32, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_tiled_kernel<T, LPI, CHORDS>, W * 32, smem);
     per_sm = std::max(per_sm, 1);
     const long long per_cta = static_cast<long long>(W) * IPW;
     const long long blocks = std::min<long long>((p + per_cta - 1) / per_cta,
                                                  static_cast<long long>(per_sm) * num_sms());
     const int c_vec = (n % 4 == 0) && aligned16(c);
-    tri_tiled_kernel<T, LPI><<<static_cast<unsigned>(blocks), W * 32, smem, st>>>(
-        static_cast<const T *>(c), static_cast<T *>(out), static_cast<int>(n), p, layout, NT, c_vec);
+    tri_tiled_kernel<T, LPI, CHORDS><<<static_cast<unsigned>(blocks), W * 32, smem, st>>>(
+        static_cast<const T *>(c), static_cast<T *>(out), chords, static_cast<int>(n), p, layout, NT, c_vec);
     return after_launch("tri_tiled_kernel");
 }
 
@@ -330,10 +380,17 @@ static int launch_tiled_t(const void *c, void *out, int64_t n, int64_t p, int la
 int launch_tri_tiled(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int lpi,
                      cudaStream_t st) {
     if (dtype == BO_F32)
-        return lpi == 16 ? launch_tiled_t<float, 16>(c, out, n, p, layout, st)
-                         : launch_tiled_t<float, 32>(c, out, n, p, layout, st);
-    return lpi == 16 ? launch_tiled_t<int32_t, 16>(c, out, n, p, layout, st)
-                     : launch_tiled_t<int32_t, 32>(c, out, n, p, layout, st);
+        return lpi == 16 ? launch_tiled_t<float, 16, false>(c, out, nullptr, n, p, layout, st)
+                         : launch_tiled_t<float, 32, false>(c, out, nullptr, n, p, layout, st);
+    return lpi == 16 ? launch_tiled_t<int32_t, 16, false>(c, out, nullptr, n, p, layout, st)
+                     : launch_tiled_t<int32_t, 32, false>(c, out, nullptr, n, p, layout, st);
+}
+
+// NEXT-1: values and the chords of an optimal triangulation (16 lanes per instance)
+int launch_tri_chords(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int dtype, int layout,
+                      cudaStream_t st) {
+    if (dtype == BO_F32) return launch_tiled_t<float, 16, true>(c, out, chords, n, p, layout, st);
+    return launch_tiled_t<int32_t, 16, true>(c, out, chords, n, p, layout, st);
 }
 
 }  // namespace bo

@@ -110,3 +110,40 @@ def test_tr2_variants_agree_full_size(variant):
     ids = np.arange(0, p, 997)
     ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 4, "float32"), oracle.ROW_WISE, nthreads=NTHREADS)
     assert np.array_equal(a.cpu().numpy()[ids].view(np.uint32), ref.view(np.uint32))
+
+
+# ------------------------------------------------------------------ NEXT-1 chords
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("n,p", [(3, 7), (4, 40), (5, 33), (8, 100), (13, 64), (16, 300), (17, 50), (33, 64),
+                                 (61, 20), (64, 130)])
+def test_chords_match_oracle(dt, layout, n, p):
+    c = bulkgen.tri_input(n, p, seed=7 * n + p, dtype=dt, layout=layout)
+    ref_v, ref_ch = oracle.bulk_opt_chords(c, layout)
+    v, ch = bo.triangulation_chords(torch.from_numpy(c).to(DEV), layout)
+    assert np.array_equal(v.cpu().numpy().view(np.uint32), ref_v.view(np.uint32))
+    assert np.array_equal(ch.cpu().numpy(), ref_ch)
+
+
+def test_chords_ties_take_the_first_k():
+    # uniform weights: every triangulation is optimal; the chosen one is fixed by the tie-break
+    n, p = 40, 8
+    w = np.zeros((n, n), dtype=np.int32)
+    for a in range(n):
+        for b in range(a + 2, n):
+            if not (a == 0 and b == n - 1):
+                w[a, b] = 3
+    c = np.broadcast_to(w, (p, n, n)).copy()
+    ref_v, ref_ch = oracle.bulk_opt_chords(c, oracle.ROW_WISE)
+    v, ch = bo.triangulation_chords(torch.from_numpy(c).to(DEV))
+    assert np.array_equal(v.cpu().numpy(), ref_v) and np.array_equal(ch.cpu().numpy(), ref_ch)
+
+
+def test_chords_tr2_full_size_sampled():
+    n, p = 64, 65536
+    c = bo.generate_tri(n, p, 4, torch.float32, bo.ROW_WISE)
+    v, ch = bo.triangulation_chords(c)
+    assert torch.equal(v.view(torch.int32), bo.triangulation(c).view(torch.int32))
+    ids = np.unique(np.r_[np.arange(0, p, 509), p - 1])
+    ref_v, ref_ch = oracle.bulk_opt_chords(bulkgen.tri_instances(n, ids, 4, "float32"), oracle.ROW_WISE)
+    assert np.array_equal(ch.cpu().numpy()[ids], ref_ch)
