@@ -1,0 +1,29 @@
+#!/usr/bin/env python
+"""Small inputs through every kernel, for compute-sanitizer (memcheck /
+racecheck / synccheck).  Run: compute-sanitizer --tool racecheck python tools/sanitize.py"""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import torch  # noqa: E402
+
+import paper_conf_ipps_tanitni14_b200 as bo  # noqa: E402
+
+for layout in (bo.ROW_WISE, bo.COLUMN_WISE):
+    for n, p in ((64, 300), (33, 129), (1024, 260)):
+        x = bo.generate_prefix(n, p, 1, torch.float32, layout)
+        vs = [bo.AUTO, bo.PS_NAIVE] + ([bo.PS_FUSED_ROW, bo.PS_WARPSCAN, bo.PS_TRANSPOSED] if layout == 0 else
+                                       [bo.PS_ACROSS])
+        for v in vs:
+            bo.prefix_sums(x, layout, v)
+    for n, p in ((16, 70), (24, 40), (64, 40)):
+        c = bo.generate_tri(n, p, 1, torch.float32, layout)
+        for v in (bo.AUTO, bo.TRI_SMEM_WARP, bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_UMM_GLOBAL) + \
+                ((bo.TRI_THREAD_REG,) if n <= 18 else ()):
+            bo.triangulation(c, layout, v)
+        bo.triangulation_chords(c, layout)
+x = torch.zeros((300, 260), dtype=torch.int32, device="cuda")
+bo.transpose(x)
+torch.cuda.synchronize()
+print("sanitize run complete")
