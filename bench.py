@@ -62,10 +62,17 @@ WORKLOADS = {
                    desc="bulk optimal triangulation int32 n=16, p=65536, column-wise weights"),
     "tr2chords": dict(seed=4, algo="tri", n=64, p=65536, dtype="float32", layout=0, variant="chords",
                       desc="NEXT-1: TR-2 values plus the chords of each optimal triangulation"),
+    "exec_bitonic_col": dict(seed=6, algo="exec", prog="bitonic", n=64, p=2 ** 20, dtype="float32", layout=1,
+                             variant=0, desc="NEXT-3: generic executor, bitonic sort n=64, column-wise (Thm 2)"),
+    "exec_bitonic_row": dict(seed=6, algo="exec", prog="bitonic", n=64, p=2 ** 20, dtype="float32", layout=0,
+                             variant=0, desc="NEXT-3: generic executor, bitonic sort n=64, row-wise (Thm 2)"),
+    "exec_prefix_col": dict(seed=2, algo="exec", prog="prefix", n=1024, p=2 ** 20, dtype="float32", layout=1,
+                            variant=0, desc="NEXT-3: generic executor running Algorithm Prefix-sums, column-wise"),
     "ps2naive_row": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=5,
                          desc="the paper's row-wise kernel (thread per instance, uncoalesced)"),
 }
-EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr2", "tr2chords", "ps2naive_col", "ps2naive_row", "tr2umm"]
+EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr2", "tr2chords", "ps2naive_col", "ps2naive_row", "tr2umm",
+          "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col"]
 L2_BYTES = 126 * 2 ** 20
 
 
@@ -78,7 +85,7 @@ def algo_bytes_per_instance(wl):
     """Algorithmic HBM bytes per instance: prefix reads
     and writes n elements; OPT reads the C(n-1,2) weights c[a][b], b-a>=2
     (the only ones Algorithm OPT touches) and writes one result."""
-    if wl["algo"] == "prefix":
+    if wl["algo"] in ("prefix", "exec"):
         return 2 * wl["n"] * 4
     n = wl["n"]
     return 4 * ((n - 1) * (n - 2) // 2 + 1)
@@ -235,6 +242,16 @@ def setup_workload(wl, rank):
     from paper_conf_ipps_tanitni14_b200 import shard
     h0, _ = shard.weak_range(p, rank)
     seed = wl["seed"]
+    if wl["algo"] == "exec":
+        from paper_conf_ipps_tanitni14_b200 import programs
+        prog = programs.bitonic_sort(n) if wl["prog"] == "bitonic" else programs.prefix_sums(n, wl["dtype"])
+        x = bo.generate_prefix(n, p, seed, dt, wl["layout"], "uniform", h0=h0)
+        pbuf = torch.empty(prog.array().shape[0] * 16, dtype=torch.uint8, device="cuda")
+
+        def fn():
+            bo.execute(prog, x, wl["layout"], prog_buf=pbuf)
+        return dict(x=x, out=x, fn=fn, seed=seed, h0=h0,
+                    variant=f"exec[{wl['prog']}: {prog.array().shape[0]} instr]")
     if wl["algo"] == "prefix":
         x = bo.generate_prefix(n, p, seed, dt, wl["layout"], "uniform", h0=h0)
         out = torch.empty_like(x)
@@ -267,7 +284,7 @@ def setup_workload(wl, rank):
 
 def input_bytes(wl):
     n, p = wl["n"], wl["p"]
-    return n * p * 4 if wl["algo"] == "prefix" else n * n * p * 4
+    return n * p * 4 if wl["algo"] in ("prefix", "exec") else n * n * p * 4
 
 
 def measure(ctx, name, steps, warmup, stream, peaks, traffic):
@@ -287,7 +304,7 @@ def measure(ctx, name, steps, warmup, stream, peaks, traffic):
            "l2": "flushed (256 MB write) between steps" if flush else "input > L2, no flush",
            "gpu_launches": launches}
     bytes_launch = algo_bytes_per_instance(wl) * wl["p"]
-    if wl["algo"] == "prefix":
+    if wl["algo"] in ("prefix", "exec"):
         gbs = bytes_launch / (ms * 1e-3) / 1e9
         res["algorithmic_GBps_per_gpu"] = gbs
         res["roofline"] = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",

@@ -134,6 +134,26 @@ int bulk_triangulation_chords(const void *c, void *out, int16_t *chords, int64_t
                               int layout, void *stream);
 
 /* ------------------------------------------------------------------------- */
+/* Generic bulk execution of an oblivious program (NEXT-3; Theorem 2,         */
+/* P:132-137).  p instances each run the same straight-line program of t      */
+/* instructions on their own memory of msize words (mem: row-wise            */
+/* [p][msize], addr j*msize + a, or column-wise [msize][p], addr a*p + j).    */
+/*   prog     : HOST int32 [t][4] = (op, x, y, z):                            */
+/*              0 LOAD r[x] <- b[y]        1 STORE b[x] <- r[y]               */
+/*              2 ADD  r[x] <- r[y] + r[z] 3 SUB   r[x] <- r[y] - r[z]        */
+/*              4 MIN  r[x] <- (r[z] < r[y] ? r[z] : r[y])                     */
+/*              5 MAX  r[x] <- (r[y] < r[z] ? r[z] : r[y])                     */
+/*              6 MOV  r[x] <- r[y]        7 CONST r[x] <- bit pattern y       */
+/*              Registers start at 0; int32 add/sub wrap mod 2^32, fp32 RN.   */
+/*              Validated on the host (registers < nregs <= 64, addresses     */
+/*              < msize): BO_EINVAL names the first bad instruction.          */
+/*   prog_dev : device buffer (16-byte aligned, >= 16*t bytes) the library    */
+/*              copies the program into, on `stream`.                         */
+/* ------------------------------------------------------------------------- */
+int bulk_execute(const int32_t *prog, int64_t t, void *prog_dev, size_t prog_dev_bytes, void *mem, int64_t msize,
+                 int64_t p, int dtype, int layout, int nregs, void *stream);
+
+/* ------------------------------------------------------------------------- */
 /* Layout transpose (row-wise <-> column-wise arrangement):        */
 /*   dst[c*rows + r] = src[r*cols + c],  0 <= r < rows, 0 <= c < cols.        */
 /* Row-wise [p][n] -> column-wise [n][p] is (rows=p, cols=n); the reverse is  */

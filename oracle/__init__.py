@@ -69,6 +69,12 @@ def lib():
         L.oracle_brute_opt_set_f64.restype = ctypes.c_double
         L.oracle_bulk_opt_chords.argtypes = [vp, vp, vp, i64, i64, i32, i32, i64, i64]
         L.oracle_bulk_opt_chords.restype = i32
+        L.oracle_exec.argtypes = [vp, i64, vp, i32]
+        L.oracle_exec.restype = i32
+        L.oracle_exec_trace.argtypes = [vp, i64, vp, i32, vp, i64]
+        L.oracle_exec_trace.restype = i64
+        L.oracle_bulk_exec.argtypes = [vp, i64, vp, i64, i64, i32, i32]
+        L.oracle_bulk_exec.restype = i32
         _lib = L
     return _lib
 
@@ -212,6 +218,40 @@ def bulk_opt_chords(c: np.ndarray, layout: int):
     rc = lib().oracle_bulk_opt_chords(_ptr(c), _ptr(out), _ptr(ch), n, p, _DT[_dtname(c)], layout, 0, p)
     assert rc == 0
     return out, ch
+
+
+# ------------------------------------------------ generic oblivious programs
+def execute(prog: np.ndarray, mem: np.ndarray) -> np.ndarray:
+    """Interpret an oblivious program (int32 [t, 4]) on one instance memory."""
+    prog = np.ascontiguousarray(prog, dtype=np.int32)
+    out = np.array(mem, copy=True, order="C")
+    rc = lib().oracle_exec(_ptr(prog), prog.shape[0], _ptr(out), _DT[_dtname(out)])
+    assert rc == 0
+    return out
+
+
+def execute_trace(prog: np.ndarray, mem: np.ndarray) -> np.ndarray:
+    prog = np.ascontiguousarray(prog, dtype=np.int32)
+    work = np.array(mem, copy=True, order="C")
+    cap = int(np.sum((prog[:, 0] == 0) | (prog[:, 0] == 1)))
+    ev = np.zeros((max(cap, 1), 3), dtype=np.int64)
+    t = lib().oracle_exec_trace(_ptr(prog), prog.shape[0], _ptr(work), _DT[_dtname(work)], _ptr(ev), cap)
+    assert t == cap
+    return ev[:t]
+
+
+def bulk_execute(prog: np.ndarray, mem: np.ndarray, layout: int) -> np.ndarray:
+    """Bulk execution (Thm 2): mem is [p, msize] row-wise or
+    [msize, p] column-wise; returns the new memory."""
+    prog = np.ascontiguousarray(prog, dtype=np.int32)
+    out = np.array(mem, copy=True, order="C")
+    if layout == ROW_WISE:
+        p, msize = out.shape
+    else:
+        msize, p = out.shape
+    rc = lib().oracle_bulk_exec(_ptr(prog), prog.shape[0], _ptr(out), msize, p, _DT[_dtname(out)], layout)
+    assert rc == 0
+    return out
 
 
 # ----------------------------------------------------------------- transpose

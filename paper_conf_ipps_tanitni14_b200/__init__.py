@@ -59,6 +59,7 @@ def lib() -> ctypes.CDLL:
             "bulk_triangulation_workspace": ([i64, i64, i32, i32, i32], sz),
             "bulk_transpose": ([vp, vp, i64, i64, sz, vp], i32),
             "bulk_triangulation_chords": ([vp, vp, vp, i64, i64, i32, i32, vp], i32),
+            "bulk_execute": ([vp, i64, vp, sz, vp, i64, i64, i32, i32, i32, vp], i32),
             "bulk_prefix_sums_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_triangulation_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_generate_prefix": ([vp, i64, i64, i64, u64, i32, i32, i32, vp], i32),
@@ -208,6 +209,27 @@ def triangulation_chords(c: torch.Tensor, layout: int = ROW_WISE, stream=None):
     _check(lib().bulk_triangulation_chords(c.data_ptr(), out.data_ptr(), chords.data_ptr() if chords.numel() else None,
                                            n, p, dt, layout, _stream(stream)))
     return out, chords
+
+
+def execute(program, mem: torch.Tensor, layout: int = COLUMN_WISE, prog_buf: torch.Tensor | None = None,
+            stream=None) -> torch.Tensor:
+    """Bulk execution of an oblivious program (NEXT-3, Theorem 2) in
+    place on mem ([p, msize] row-wise or [msize, p] column-wise).  `program`
+    is a programs.Program or an int32 array [t, 4] (then nregs = 64)."""
+    import numpy as np
+    _need_cuda(mem)
+    if hasattr(program, "array"):
+        code, nregs = program.array(), program.nregs
+    else:
+        code, nregs = np.asarray(program, dtype=np.int32).reshape(-1, 4), 64
+    code = np.ascontiguousarray(code, dtype=np.int32)
+    t = code.shape[0]
+    msize, p = _shape_np(mem, layout)
+    if prog_buf is None:
+        prog_buf = torch.empty(max(t, 1) * 16, dtype=torch.uint8, device=mem.device)
+    _check(lib().bulk_execute(code.ctypes.data, t, prog_buf.data_ptr(), prog_buf.numel(), mem.data_ptr(), msize, p,
+                              _dtype_code(mem), layout, nregs, _stream(stream)))
+    return mem   # pageable H2D copies return once the host program is staged
 
 
 def triangulation_host(c_host: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO,

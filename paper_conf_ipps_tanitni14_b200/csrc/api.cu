@@ -65,6 +65,8 @@ size_t tri_workspace(int64_t n, int64_t p, int variant);
 int launch_gen_prefix(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
 int launch_gen_tri(void *, int64_t, int64_t, int64_t, uint64_t, int, int, cudaStream_t);
 int launch_checksum(const void *, int64_t, int64_t, int64_t, int, uint64_t *, cudaStream_t);
+int launch_exec(const void *prog, int64_t t, void *mem, int64_t msize, int64_t p, int dtype, int layout, int nregs,
+                cudaStream_t st);
 
 static constexpr int64_t kMaxElems = int64_t(1) << 40;
 
@@ -207,6 +209,41 @@ int bulk_triangulation(const void *c, void *out, int64_t n, int64_t p, int dtype
     if (need > 0 && (!workspace || workspace_bytes < need))
         return fail(BO_EINVAL, "triangulation: workspace too small (need " + std::to_string(need) + " bytes)");
     return tri_dispatch(c, out, n, p, dtype, layout, v, workspace, static_cast<cudaStream_t>(stream));
+}
+
+int bulk_execute(const int32_t *prog, int64_t t, void *prog_dev, size_t prog_dev_bytes, void *mem, int64_t msize,
+                 int64_t p, int dtype, int layout, int nregs, void *stream) {
+    t_err.clear();
+    if (t < 0 || msize < 0 || p < 0) return fail(BO_EINVAL, "execute: t, msize and p must be >= 0");
+    if (!valid_dtype(dtype) || !valid_layout(layout)) return fail(BO_EINVAL, "execute: bad dtype or layout");
+    if (nregs < 1 || nregs > 64) return fail(BO_EINVAL, "execute: need 1 <= nregs <= 64");
+    if (msize > 0 && p > kMaxElems / msize) return fail(BO_EINVAL, "execute: msize*p too large");
+    if (t == 0 || p == 0) return BO_OK;
+    if (!prog || !mem) return fail(BO_EINVAL, "execute: NULL pointer");
+    if (!prog_dev || prog_dev_bytes < static_cast<size_t>(t) * 16 || !aligned16(prog_dev))
+        return fail(BO_EINVAL, "execute: device program buffer must be 16-byte aligned and >= 16*t bytes");
+    // the program is validated here, on the host: every register < nregs and
+    // every address < msize, so the kernel never leaves the instance memory
+    for (int64_t i = 0; i < t; ++i) {
+        const int32_t op = prog[4 * i], x = prog[4 * i + 1], y = prog[4 * i + 2], z = prog[4 * i + 3];
+        auto reg = [&](int32_t r) { return r >= 0 && r < nregs; };
+        auto adr = [&](int32_t a) { return a >= 0 && a < msize; };
+        bool ok;
+        switch (op) {
+            case 0: ok = reg(x) && adr(y); break;
+            case 1: ok = adr(x) && reg(y); break;
+            case 2: case 3: case 4: case 5: ok = reg(x) && reg(y) && reg(z); break;
+            case 6: ok = reg(x) && reg(y); break;
+            case 7: ok = reg(x); break;
+            default: ok = false;
+        }
+        if (!ok) return fail(BO_EINVAL, "execute: bad instruction " + std::to_string(i));
+    }
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    int rc = cuda_check(cudaMemcpyAsync(prog_dev, prog, static_cast<size_t>(t) * 16, cudaMemcpyHostToDevice, st),
+                        "execute: program upload");
+    if (rc) return rc;
+    return launch_exec(prog_dev, t, mem, msize, p, dtype, layout, nregs, st);
 }
 
 int bulk_triangulation_chords(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int dtype,

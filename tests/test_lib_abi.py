@@ -114,3 +114,16 @@ def test_product_package_never_imports_oracle():
                 text = open(os.path.join(dirpath, f), errors="replace").read()
                 assert "import oracle" not in text and "from oracle" not in text, f
                 assert "oracle.c" not in text and "liboracle" not in text, f
+
+
+def test_execute_validates_program_on_host(L):
+    import numpy as np
+    p = ctypes.c_void_p(4096)           # 16-byte aligned, never dereferenced
+    good = np.array([[0, 0, 3, 0], [1, 3, 0, 0]], dtype=np.int32)
+    for bad in ([[0, 0, 8, 0]], [[0, 5, 0, 0]], [[9, 0, 0, 0]], [[2, 0, 1, 70]]):
+        prog = np.array(bad, dtype=np.int32)
+        assert L.bulk_execute(prog.ctypes.data, 1, p, 16, p, 8, 4, 0, 0, 4, None) == -1
+        assert b"bad instruction 0" in L.bulk_last_error()
+    assert L.bulk_execute(good.ctypes.data, 2, p, 16, p, 8, 4, 0, 0, 4, None) == -1   # program buffer too small
+    assert L.bulk_execute(good.ctypes.data, 2, p, 32, p, 8, 4, 0, 0, 0, None) == -1   # nregs = 0
+    assert L.bulk_execute(good.ctypes.data, 0, p, 32, p, 8, 4, 0, 0, 4, None) == 0    # empty program
