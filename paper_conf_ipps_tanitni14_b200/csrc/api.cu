@@ -55,7 +55,8 @@ bool make_tmap_2d(CUtensorMap *map, const void *base, uint64_t rows, uint64_t co
 int launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, cudaStream_t st);
 int prefix_dispatch(const void *src, void *dst, int64_t n, int64_t p, int dtype, int layout, int variant,
                     void *ws, cudaStream_t st);
-int resolve_prefix_variant(int64_t n, int64_t p, int layout, int variant, const void *src, const void *dst);
+int resolve_prefix_variant(int64_t n, int64_t p, int dtype, int layout, int variant, const void *src,
+                           const void *dst);
 int tri_dispatch(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int variant, void *ws,
                  cudaStream_t st);
 int resolve_tri_variant(int64_t n, int64_t p, int dtype, int layout, int variant);
@@ -165,13 +166,11 @@ const char *bulk_version(void) { return "bulkobl 0.1 (sm_100a)"; }
 
 int bulk_prefix_sums_variant(int64_t n, int64_t p, int dtype, int layout, int variant, const void *src,
                              const void *dst) {
-    (void)dtype;
-    return resolve_prefix_variant(n, p, layout, variant, src, dst);
+    return resolve_prefix_variant(n, p, dtype, layout, variant, src, dst);
 }
 
 size_t bulk_prefix_sums_workspace(int64_t n, int64_t p, int dtype, int layout, int variant) {
-    (void)dtype;
-    return prefix_ws(n, p, resolve_prefix_variant(n, p, layout, variant, nullptr, nullptr));
+    return prefix_ws(n, p, resolve_prefix_variant(n, p, dtype, layout, variant, nullptr, nullptr));
 }
 
 int bulk_prefix_sums(const void *src, void *dst, int64_t n, int64_t p, int dtype, int layout, int variant,
@@ -180,7 +179,7 @@ int bulk_prefix_sums(const void *src, void *dst, int64_t n, int64_t p, int dtype
     int rc = check_prefix_args(src, dst, n, p, dtype, layout, variant);
     if (rc) return rc;
     if (n * p == 0) return BO_OK;
-    const int v = resolve_prefix_variant(n, p, layout, variant, src, dst);
+    const int v = resolve_prefix_variant(n, p, dtype, layout, variant, src, dst);
     const size_t need = prefix_ws(n, p, v);
     if (need > 0 && (!workspace || workspace_bytes < need))
         return fail(BO_EINVAL, "prefix: workspace too small (need " + std::to_string(need) + " bytes)");
@@ -301,7 +300,7 @@ int bulk_prefix_sums_host(const void *h_src, void *h_dst, int64_t n, int64_t p, 
     int rc = check_prefix_args(h_src, h_dst, n, p, dtype, layout, variant);
     if (rc) return rc;
     if (n * p == 0) return BO_OK;
-    const int v = resolve_prefix_variant(n, p, layout, variant, nullptr, nullptr);
+    const int v = resolve_prefix_variant(n, p, dtype, layout, variant, nullptr, nullptr);
     const int64_t ch = host_chunk(p);
     const size_t data_bytes = static_cast<size_t>(n) * p * 4;
     const size_t ws_chunk = prefix_ws(n, ch, v);

@@ -93,6 +93,8 @@ def test_workspace_and_variant_queries(L):
     assert bo.prefix_sums_workspace(1024, 100, bo.F32, bo.ROW_WISE) == 0
     assert bo.prefix_sums_variant(1024, 100, bo.F32, bo.ROW_WISE) == bo.PS_FUSED_ROW
     assert bo.prefix_sums_variant(1024, 100, bo.F32, bo.COLUMN_WISE) == bo.PS_ACROSS
+    assert bo.prefix_sums_variant(32, 1024, bo.I32, bo.ROW_WISE) == bo.PS_WARPSCAN     # int32: exact, latency win
+    assert bo.prefix_sums_variant(32, 2 ** 22, bo.I32, bo.ROW_WISE) == bo.PS_FUSED_ROW
     assert bo.triangulation_variant(16, 100, bo.I32, bo.ROW_WISE) == bo.TRI_THREAD_REG
     assert bo.triangulation_variant(64, 100, bo.F32, bo.ROW_WISE) == bo.TRI_TILED_HALF
     assert bo.triangulation_variant(100, 100, bo.F32, bo.ROW_WISE) == bo.TRI_SMEM_WARP
