@@ -93,6 +93,9 @@ __device__ __forceinline__ void cp_async16(void *dst, const void *src, bool pred
         "l"(src), "r"(static_cast<int>(pred))
         : "memory");
 }
+__device__ __forceinline__ void cp_async4(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
 // S[u][v] = min(S[u][v], min_w A[u].w + B[w].v) for one 4-wide k chunk
@@ -160,8 +163,9 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
     const long long nn = static_cast<long long>(n) * n;
     const int last_chunk = (n - 1) >> 2;
 
-    for (long long h = (static_cast<long long>(blockIdx.x) * warps_per_cta + warp) * IPW + slot;
-         h - slot < p; h += inst_stride) {
+    const int ninst = warps_per_cta * IPW;              // consecutive instances per CTA pass
+    for (long long base = static_cast<long long>(blockIdx.x) * ninst; base < p; base += inst_stride) {
+        const long long h = base + warp * IPW + slot;
         const bool live = h < p;
         // ------------------------------------------------ 1. c -> upper table
         // Only the weights Algorithm OPT reads (b >= a+2) are fetched.
@@ -184,11 +188,27 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
                 }
             }
             tt::cp_async_wait_all();
+        } else if (layout == BO_COLUMN_WISE) {
+            // Column-wise weights c[(a*n+b)*p + h]: the whole CTA loads the
+            // weights of its `ninst` consecutive instances together, instance index
+            // fastest, so each warp request covers whole 32-byte sectors.
+            __syncthreads();                                // every table of the CTA is free
+            T *Z0 = reinterpret_cast<T *>(smem_raw);
+            for (int a = 0; a < n - 2; ++a) {
+                const int L = n - a - 2;                    // cells (a, a+2 .. n-1)
+                const long long row0 = static_cast<long long>(a) * n + a + 2;
+                for (int idx = threadIdx.x; idx < L * ninst; idx += blockDim.x) {
+                    const int q = idx % ninst, b = a + 2 + idx / ninst;
+                    if (base + q < p)
+                        tt::cp_async4(Z0 + static_cast<size_t>(q) * words + tt::xoff(a, b),
+                                      c + (row0 + (b - a - 2)) * p + base + q);
+                }
+            }
+            tt::cp_async_wait_all();
+            __syncthreads();
         } else if (live) {
             for (int a = 0; a < n - 2; ++a)
-                for (int b = a + 2 + li; b < n; b += LPI)
-                    Z[tt::xoff(a, b)] = __ldg(c + (layout == BO_ROW_WISE ? h * nn + static_cast<long long>(a) * n + b
-                                                                      : (static_cast<long long>(a) * n + b) * p + h));
+                for (int b = a + 2 + li; b < n; b += LPI) Z[tt::xoff(a, b)] = __ldg(c + h * nn + static_cast<long long>(a) * n + b);
         }
         __syncwarp();
 
@@ -356,7 +376,8 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
     for (int w = 1; w <= 4; ++w) {
         const size_t per_cta = w * IPW * per_inst + 1024;
         const int resident = static_cast<int>((227 * 1024) / per_cta) * w;
-        if (resident > best) best = resident, W = w;
+        // column-wise weights: prefer 4 warps (8+ consecutive instances = whole sectors)
+        if (resident > best || (layout == BO_COLUMN_WISE && resident == best)) best = resident, W = w;
     }
     const size_t smem = W * IPW * per_inst;
     static bool attr = [] {
