@@ -487,7 +487,10 @@ def run_ours(args, ctx):
             torch.cuda.empty_cache()
         line["extras"] = ex
     if args.e2e:
-        line["e2e"] = e2e(ctx, name, max(2, min(args.steps, 5)), 1)
+        try:
+            line["e2e"] = e2e(ctx, name, max(2, min(args.steps, 5)), 1)
+        except Exception as exc:                    # e.g. pinned host memory exhausted at 8 ranks
+            line["e2e"] = {"error": repr(exc)}
     if args.cpu_baseline and ctx.rank == 0 and ctx.world == 1:
         line["cpu_baseline"] = cpu_baseline(ctx, name, st)
     elif args.cpu_baseline:
