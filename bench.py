@@ -393,13 +393,19 @@ def e2e(ctx, name, steps, warmup):
     if wl["algo"] != "prefix":
         return None
     shape = (p, n) if wl["layout"] == 0 else (n, p)
-    dev = bo.generate_prefix(n, p, wl["seed"], dt, wl["layout"], "uniform", h0=ctx.rank * p)
-    h_in = torch.empty(shape, dtype=dt, pin_memory=True)
-    h_in.copy_(dev)
-    h_out = torch.empty(shape, dtype=dt, pin_memory=True)
-    del dev
-    dbuf = torch.empty(n * p * 4, dtype=torch.uint8, device="cuda")
-    torch.cuda.synchronize()
+    err = None
+    try:
+        dev = bo.generate_prefix(n, p, wl["seed"], dt, wl["layout"], "uniform", h0=ctx.rank * p)
+        h_in = torch.empty(shape, dtype=dt, pin_memory=True)
+        h_in.copy_(dev)
+        h_out = torch.empty(shape, dtype=dt, pin_memory=True)
+        del dev
+        dbuf = torch.empty(n * p * 4, dtype=torch.uint8, device="cuda")
+        torch.cuda.synchronize()
+    except Exception as exc:        # agree across ranks before any barrier
+        err = repr(exc)
+    if ctx.max(1.0 if err else 0.0) > 0:
+        raise RuntimeError(err or "e2e buffers could not be allocated on another rank")
     stream = torch.cuda.current_stream()
 
     def fn():
