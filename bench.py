@@ -60,6 +60,8 @@ WORKLOADS = {
                    desc="the paper's column-wise UMM kernel on TR-2"),
     "tr1col": dict(seed=3, algo="tri", n=16, p=65536, dtype="int32", layout=1, variant=0,
                    desc="bulk optimal triangulation int32 n=16, p=65536, column-wise weights"),
+    "tr512": dict(seed=7, algo="tri", n=512, p=1024, dtype="float32", layout=0, variant=0,
+                  desc="NEXT-2: the paper's 512-gons at its largest p (P:251), fp32, row-wise"),
     "tr2chords": dict(seed=4, algo="tri", n=64, p=65536, dtype="float32", layout=0, variant="chords",
                       desc="NEXT-1: TR-2 values plus the chords of each optimal triangulation"),
     "exec_bitonic_col": dict(seed=6, algo="exec", prog="bitonic", n=64, p=2 ** 20, dtype="float32", layout=1,
@@ -71,7 +73,7 @@ WORKLOADS = {
     "ps2naive_row": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=5,
                          desc="the paper's row-wise kernel (thread per instance, uncoalesced)"),
 }
-EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr2", "tr2chords", "ps2naive_col", "ps2naive_row", "tr2umm",
+EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr2", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
           "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col"]
 L2_BYTES = 126 * 2 ** 20
 

@@ -78,8 +78,12 @@ typedef enum {
     BO_TRI_THREAD_REG = 18, /* thread per instance, M in registers (3 <= n <= 18) */
     BO_TRI_TILED = 19,      /* warp per instance, M in shared memory, 4x4 register
                                tiles (min-plus blocked product), 5 <= n <= 64     */
-    BO_TRI_TILED_HALF = 20  /* as BO_TRI_TILED with 16 lanes per instance (two
+    BO_TRI_TILED_HALF = 20, /* as BO_TRI_TILED with 16 lanes per instance (two
                                instances per warp)                                 */
+    BO_TRI_TILED_GLOBAL = 21 /* CTA per instance, same blocked algorithm, table in a
+                               per-CTA global workspace slot kept L2-resident
+                               (large n, e.g. 512-gons); workspace
+                               min(p, #SMs) * 16 * (2T^2 + 3T) bytes, T = ceil(n/4) */
 } bo_variant;
 
 /* ------------------------------------------------------------------------- */

@@ -237,6 +237,9 @@ tri_smem_warp(const T *__restrict__ c, T *__restrict__ out, int n, long long p, 
 
 // ------------------------------------------------------------------- host
 int tiled_supported(int64_t n);
+size_t tiled_global_workspace(int64_t n, int64_t p);
+int launch_tri_tiled_global(const void *c, void *out, void *ws, int64_t n, int64_t p, int dtype, int layout,
+                            cudaStream_t st);
 int launch_tri_tiled(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int lpi,
                      cudaStream_t st);
 
@@ -252,12 +255,12 @@ int resolve_tri_variant(int64_t n, int64_t p, int dtype, int layout, int variant
     if (variant != BO_AUTO) return variant;
     if (n <= 16) return BO_TRI_THREAD_REG;
     if (tiled_supported(n)) return BO_TRI_TILED_HALF;   // 16 lanes per instance: faster at every n measured
-    if (smem_per_instance(n) <= 200 * 1024) return BO_TRI_SMEM_WARP;
-    return BO_TRI_UMM_GLOBAL;
+    return BO_TRI_TILED_GLOBAL;
 }
 
 size_t tri_workspace(int64_t n, int64_t p, int variant) {
     if (variant == BO_TRI_UMM_GLOBAL) return static_cast<size_t>(n - 1) * (n - 1) * p * 4;
+    if (variant == BO_TRI_TILED_GLOBAL) return tiled_global_workspace(n, p);
     return 0;
 }
 
@@ -351,6 +354,9 @@ static int run_tri(const void *c, void *out, int64_t n, int64_t p, int layout, i
             if (!tiled_supported(n)) return fail(BO_EUNSUPPORTED, "triangulation TILED supports 5 <= n <= 64");
             return launch_tri_tiled(c, out, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout,
                                     variant == BO_TRI_TILED ? 32 : 16, st);
+        case BO_TRI_TILED_GLOBAL:
+            return launch_tri_tiled_global(c, out, ws, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout,
+                                           st);
         default:
             return fail(BO_EINVAL, "triangulation: unknown variant");
     }

@@ -414,4 +414,148 @@ int launch_tri_chords(const void *c, void *out, int16_t *chords, int64_t n, int6
     return launch_tiled_t<int32_t, 16, true>(c, out, chords, n, p, layout, st);
 }
 
+// ---------------------------------------------------------------------------
+// TILED_GLOBAL (NEXT-2, large polygons, e.g. the paper's 512-gons):
+// the same blocked algorithm with one CTA per instance and the chunk-column
+// table in a global workspace slot per CTA (grid = #SMs, so the working set
+// stays L2-resident: 530 KB x 148 = 78 MB at n = 512).  __syncthreads orders
+// the tile-diagonals; a tile's split lanes stay inside one warp (s <= 32).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ int split_log2_cta(int t, int D, int threads) {
+    int ls = 0;
+    while ((2 << ls) * t <= threads && (1 << ls) < D - 1 && (2 << ls) <= 32) ++ls;
+    return ls;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(512, 1)
+tri_tiled_global_kernel(const T *__restrict__ c, T *__restrict__ out, T *ws, int n, long long p, int layout, int NT,
+                        int c_vec) {
+    using Op = tt::Ops<T>;
+    using T4 = typename tt::V4<T>::type;
+    using tt::xc;
+    const long long words = 4LL * tt::colbase(NT);
+    T *Z = ws + static_cast<long long>(blockIdx.x) * words;
+    const int tid = threadIdx.x, nthr = blockDim.x;
+    const long long nn = static_cast<long long>(n) * n;
+    for (long long i = tid; i < words; i += nthr) Z[i] = T(0);      // padding stays finite
+    for (long long h = blockIdx.x; h < p; h += gridDim.x) {
+        __syncthreads();
+        // 1. weights b >= a+2 -> upper table
+        if (layout == BO_ROW_WISE && c_vec) {
+            const T4 *src = reinterpret_cast<const T4 *>(c + h * nn);
+            for (int idx = tid; idx < (n - 2) * NT; idx += nthr) {
+                const int a = idx / NT, m = idx - a * NT;
+                if (m >= ((a + 2) >> 2)) *reinterpret_cast<T4 *>(Z + xc(a, m)) = __ldg(src + static_cast<long long>(a) * (n / 4) + m);
+            }
+        } else {
+            for (int a = 0; a < n - 2; ++a)
+                for (int b = a + 2 + tid; b < n; b += nthr) {
+                    const long long e = static_cast<long long>(a) * n + b;
+                    Z[tt::xoff(a, b)] = __ldg(c + (layout == BO_ROW_WISE ? h * nn + e : e * p + h));
+                }
+        }
+        __syncthreads();
+        // 2. D = 0
+        for (int I = tid; I < NT; I += nthr) {
+            T *r0 = Z + xc(4 * I, I);
+            const T4 c0 = tt::ld4(r0), c1 = tt::ld4(r0 + 4);
+            const T z = T(0);
+            const T t02 = Op::add(Op::add(z, z), c0.z);
+            const T t13 = Op::add(Op::add(z, z), c1.w);
+            const T t03 = Op::add(Op::min(Op::add(z, t13), Op::add(t02, z)), c0.w);
+            tt::st4(r0, z, z, t02, t03);
+            tt::st4(r0 + 4, z, z, z, t13);
+            tt::st4(r0 + 8, z, z, z, z);
+            tt::st4(r0 + 12, z, z, z, z);
+        }
+        __syncthreads();
+        // 3. tile-diagonals
+        for (int D = 1; D < NT; ++D) {
+            const int t = NT - D;
+            const int ls = split_log2_cta(t, D, nthr);
+            const int s = 1 << ls;
+            for (int base = 0; base < t * s; base += nthr) {       // more tiles than threads: loop
+                const int slot = base + tid;
+                const int I = slot >> ls, q = slot & (s - 1);
+                const bool act = I < t;
+                const int J = I + D;
+                T acc[4][4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u)
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) acc[u][v] = Op::inf();
+                if (act) {
+                    for (int m = I + 1 + q; m < J; m += s) {
+                        const T *pa = Z + xc(4 * I, m), *pb = Z + xc(4 * m, J);
+                        T4 A[4], B[4];
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) A[u] = tt::ld4(pa + 4 * u), B[u] = tt::ld4(pb + 4 * u);
+                        tt::minplus_chunk(acc, A, B);
+                    }
+                }
+                for (int off = 1; off < s; off <<= 1)
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+#pragma unroll
+                        for (int v = 0; v < 4; ++v)
+                            acc[u][v] = Op::min(acc[u][v], __shfl_xor_sync(0xffffffffu, acc[u][v], off));
+                if (act && q == 0) {
+                    T *ta = Z + xc(4 * I, I), *tb = Z + xc(4 * J, J), *tc = Z + xc(4 * I, J);
+                    T A[4][4], Bd[4][4], C[4][4];
+#pragma unroll
+                    for (int r = 0; r < 4; ++r) {
+                        const T4 x = tt::ld4(ta + 4 * r), y = tt::ld4(tb + 4 * r), w = tt::ld4(tc + 4 * r);
+                        A[r][0] = x.x; A[r][1] = x.y; A[r][2] = x.z; A[r][3] = x.w;
+                        Bd[r][0] = y.x; Bd[r][1] = y.y; Bd[r][2] = y.z; Bd[r][3] = y.w;
+                        C[r][0] = w.x; C[r][1] = w.y; C[r][2] = w.z; C[r][3] = w.w;
+                    }
+                    T tt_[4][4];
+#pragma unroll
+                    for (int u = 3; u >= 0; --u)
+#pragma unroll
+                        for (int v = 0; v < 4; ++v) {
+                            T sv = acc[u][v];
+#pragma unroll
+                            for (int w = u + 1; w < 4; ++w) sv = Op::addmin(A[u][w], tt_[w][v], sv);
+#pragma unroll
+                            for (int w = 0; w < v; ++w) sv = Op::addmin(tt_[u][w], Bd[w][v], sv);
+                            tt_[u][v] = Op::add(sv, C[u][v]);
+                            if (u == 3 && v == 0 && D == 1) tt_[u][v] = T(0);
+                        }
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) tt::st4(tc + 4 * u, tt_[u][0], tt_[u][1], tt_[u][2], tt_[u][3]);
+                }
+            }
+            __syncthreads();
+        }
+        if (tid == 0) out[h] = Z[tt::xoff(0, n - 1)];
+    }
+}
+
+int tiled_global_threads(int64_t n) { return n >= 256 ? 512 : 256; }
+
+size_t tiled_global_workspace(int64_t n, int64_t p) {
+    const int NT = static_cast<int>((n + 3) / 4);
+    const long long grid = std::min<long long>(p, num_sms());
+    return static_cast<size_t>(grid) * 4 * tt::colbase(NT) * 4;
+}
+
+int launch_tri_tiled_global(const void *c, void *out, void *ws, int64_t n, int64_t p, int dtype, int layout,
+                            cudaStream_t st) {
+    const int NT = static_cast<int>((n + 3) / 4);
+    const long long grid = std::min<long long>(p, num_sms());
+    const int threads = tiled_global_threads(n);
+    const int c_vec = (n % 4 == 0) && aligned16(c);
+    if (dtype == BO_F32)
+        tri_tiled_global_kernel<float><<<static_cast<unsigned>(grid), threads, 0, st>>>(
+            static_cast<const float *>(c), static_cast<float *>(out), static_cast<float *>(ws), static_cast<int>(n), p,
+            layout, NT, c_vec);
+    else
+        tri_tiled_global_kernel<int32_t><<<static_cast<unsigned>(grid), threads, 0, st>>>(
+            static_cast<const int32_t *>(c), static_cast<int32_t *>(out), static_cast<int32_t *>(ws),
+            static_cast<int>(n), p, layout, NT, c_vec);
+    return after_launch("tri_tiled_global_kernel");
+}
+
 }  // namespace bo

@@ -18,7 +18,7 @@ NTHREADS = os.cpu_count() or 1
 
 
 def _variants(n):
-    v = [bo.AUTO, bo.TRI_UMM_GLOBAL, bo.TRI_SMEM_WARP]
+    v = [bo.AUTO, bo.TRI_UMM_GLOBAL, bo.TRI_SMEM_WARP, bo.TRI_TILED_GLOBAL]
     if n <= 18:
         v.append(bo.TRI_THREAD_REG)
     if 5 <= n <= 64:
@@ -98,7 +98,8 @@ def test_tr2_full_config(layout):
     assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32))
 
 
-@pytest.mark.parametrize("variant", [bo.TRI_SMEM_WARP, bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_UMM_GLOBAL])
+@pytest.mark.parametrize("variant", [bo.TRI_SMEM_WARP, bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_TILED_GLOBAL,
+                                     bo.TRI_UMM_GLOBAL])
 def test_tr2_variants_agree_full_size(variant):
     n, p = 64, 65536
     c = bo.generate_tri(n, p, 4, torch.float32, bo.ROW_WISE)
@@ -147,3 +148,23 @@ def test_chords_tr2_full_size_sampled():
     ids = np.unique(np.r_[np.arange(0, p, 509), p - 1])
     ref_v, ref_ch = oracle.bulk_opt_chords(bulkgen.tri_instances(n, ids, 4, "float32"), oracle.ROW_WISE)
     assert np.array_equal(ch.cpu().numpy()[ids], ref_ch)
+
+
+# ------------------------------------------------ NEXT-2: the paper's large polygons
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("n,p", [(256, 5), (512, 3), (130, 20)])
+def test_large_polygons_match_oracle(dt, layout, n, p):
+    c = bulkgen.tri_input(n, p, seed=n + p, dtype=dt, layout=layout)
+    ref = oracle.bulk_opt(c, layout, nthreads=NTHREADS)
+    got = bo.triangulation(torch.from_numpy(c).to(DEV), layout).cpu().numpy()       # AUTO -> TILED_GLOBAL
+    assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+
+
+def test_512gon_paper_config_sampled():
+    n, p = 512, 1024                     # the paper's largest 512-gon run
+    c = bo.generate_tri(n, p, 7, torch.float32, bo.ROW_WISE)
+    got = bo.triangulation(c).cpu().numpy()
+    ids = np.array([0, 511, 1023])
+    ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 7, "float32"), oracle.ROW_WISE, nthreads=NTHREADS)
+    assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32))
