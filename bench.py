@@ -60,6 +60,10 @@ WORKLOADS = {
                    desc="the paper's column-wise UMM kernel on TR-2"),
     "tr1col": dict(seed=3, algo="tri", n=16, p=65536, dtype="int32", layout=1, variant=0,
                    desc="bulk optimal triangulation int32 n=16, p=65536, column-wise weights"),
+    "tr1packed": dict(seed=3, algo="tri", n=16, p=65536, dtype="int32", layout=2, variant=0,
+                      desc="NEXT-4: TR-1 with packed weights (only the C(n-1,2) weights OPT reads)"),
+    "tr2packed": dict(seed=4, algo="tri", n=64, p=65536, dtype="float32", layout=2, variant=0,
+                      desc="NEXT-4: TR-2 with packed weights"),
     "tr512": dict(seed=7, algo="tri", n=512, p=1024, dtype="float32", layout=0, variant=0,
                   desc="NEXT-2: the paper's 512-gons at its largest p (P:251), fp32, row-wise"),
     "tr2chords": dict(seed=4, algo="tri", n=64, p=65536, dtype="float32", layout=0, variant="chords",
@@ -73,7 +77,7 @@ WORKLOADS = {
     "ps2naive_row": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=5,
                          desc="the paper's row-wise kernel (thread per instance, uncoalesced)"),
 }
-EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr2", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
+EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr1packed", "tr2", "tr2packed", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
           "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col"]
 L2_BYTES = 126 * 2 ** 20
 
@@ -286,7 +290,9 @@ def setup_workload(wl, rank):
 
 def input_bytes(wl):
     n, p = wl["n"], wl["p"]
-    return n * p * 4 if wl["algo"] in ("prefix", "exec") else n * n * p * 4
+    if wl["algo"] in ("prefix", "exec"):
+        return n * p * 4
+    return ((n - 1) * (n - 2) // 2 if wl["layout"] >= 2 else n * n) * p * 4
 
 
 def measure(ctx, name, steps, warmup, stream, peaks, traffic):

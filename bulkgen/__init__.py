@@ -37,6 +37,8 @@ M2 = np.uint64(0x94D049BB133111EB)
 
 ROW_WISE = 0     # [p][n]: b_j[i] at j*n + i
 COLUMN_WISE = 1  # [n][p]: b_j[i] at i*p + j
+PACKED_ROW = 2   # triangulation weights: [p][K], only b-a >= 2, row by row (NEXT-4)
+PACKED_COLUMN = 3  # [K][p]
 
 
 def mix64(z: np.ndarray) -> np.ndarray:
@@ -112,12 +114,26 @@ def tri_instances(n: int, ids, seed: int, dtype: str = "float32") -> np.ndarray:
     return np.ascontiguousarray(_tri_values(n, u64(seed, h, e), dtype))
 
 
+def packed_pairs(n: int):
+    """(a, b) pairs of the packed layouts, in storage order: rows a = 0..n-3,
+    b = a+2..n-1 (index k(a,b) = a(n-2) - a(a-1)/2 + (b-a-2))."""
+    return [(a, b) for a in range(n - 2) for b in range(a + 2, n)]
+
+
 def tri_input(n: int, p: int, seed: int, dtype: str = "float32", layout: int = ROW_WISE,
               h0: int = 0) -> np.ndarray:
-    """Dense chord weights: ROW_WISE [p, n, n] (c[h*n*n + a*n + b]),
-    COLUMN_WISE [n, n, p] (c[(a*n + b)*p + h])."""
+    """Chord weights: ROW_WISE [p, n, n] (c[h*n*n + a*n + b]), COLUMN_WISE
+    [n, n, p] (c[(a*n + b)*p + h]), PACKED_ROW [p, K], PACKED_COLUMN [K, p]."""
     v = tri_instances(n, np.arange(h0, h0 + p), seed, dtype)
-    return v if layout == ROW_WISE else np.ascontiguousarray(np.moveaxis(v, 0, 2))
+    if layout == ROW_WISE:
+        return v
+    if layout == COLUMN_WISE:
+        return np.ascontiguousarray(np.moveaxis(v, 0, 2))
+    pr = packed_pairs(n)
+    a = np.array([x for x, _ in pr], dtype=np.int64)
+    b = np.array([y for _, y in pr], dtype=np.int64)
+    pk = np.ascontiguousarray(v[:, a, b]) if len(pr) else np.zeros((p, 0), dtype=v.dtype)
+    return pk if layout == PACKED_ROW else np.ascontiguousarray(pk.T)
 
 
 def checksum(values: np.ndarray, layout: int = ROW_WISE, h0: int = 0) -> int:

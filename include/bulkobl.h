@@ -49,7 +49,12 @@ typedef enum {
 
 typedef enum {
     BO_ROW_WISE = 0,     /* p rows x n columns: b_j[i] at address j*n + i   */
-    BO_COLUMN_WISE = 1   /* n rows x p columns: b_j[i] at address i*p + j   */
+    BO_COLUMN_WISE = 1,  /* n rows x p columns: b_j[i] at address i*p + j   */
+    /* triangulation weights only (NEXT-4): just the K = (n-1)(n-2)/2 weights   */
+    /* c[a][b], b - a >= 2, that Algorithm OPT reads, row by row:        */
+    /* k(a,b) = a(n-2) - a(a-1)/2 + (b-a-2).                                     */
+    BO_PACKED_ROW = 2,   /* c[h*K + k]                                             */
+    BO_PACKED_COLUMN = 3 /* c[k*p + h]                                             */
 } bo_layout;
 
 typedef enum { BO_I32 = 0, BO_F32 = 1 } bo_dtype;
@@ -110,7 +115,8 @@ size_t bulk_prefix_sums_workspace(int64_t n, int64_t p, int dtype, int layout, i
 /* to 0 to get the pure chord total).  Only entries c[a][b] with b-a >= 2 are */
 /* read.                                                                       */
 /*   c   : device, dense n x n weights per instance.  Row-wise:               */
-/*         c[h*n*n + a*n + b];  column-wise: c[(a*n + b)*p + h]. */
+/*         c[h*n*n + a*n + b];  column-wise: c[(a*n + b)*p + h], */
+/*         or packed (BO_PACKED_ROW / BO_PACKED_COLUMN, see bo_layout).       */
 /*   out : device, p elements of dtype.                                       */
 /*   n >= 3 (n < 3 is BO_EINVAL), p >= 0; n <= 4096.                          */
 /*   int32 weights must satisfy |c| < 2^31 / (2(n-2)) (no overflow); fp32     */

@@ -22,7 +22,7 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 CFLAGS = ["-O2", "-fno-fast-math", "-ffp-contract=off", "-std=c11", "-fPIC", "-shared",
           "-Wall", "-pthread"]
 
-ROW_WISE, COLUMN_WISE = 0, 1
+ROW_WISE, COLUMN_WISE, PACKED_ROW, PACKED_COLUMN = 0, 1, 2, 3
 _DT = {"int32": 0, "float32": 1}
 
 
@@ -128,6 +128,19 @@ def bulk_prefix_sums(data: np.ndarray, layout: int, nthreads: int = 1,
 
 
 # ---------------------------------------------------------------------- OPT
+def _tri_pn(c: np.ndarray, layout: int):
+    """(p, n) of a weight array: [p,n,n] / [n,n,p] dense, [p,K] / [K,p] packed
+    with K = (n-1)(n-2)/2 (the weights Algorithm OPT reads)."""
+    if layout == ROW_WISE:
+        return c.shape[0], c.shape[1]
+    if layout == COLUMN_WISE:
+        return c.shape[2], c.shape[0]
+    K = c.shape[1] if layout == PACKED_ROW else c.shape[0]
+    n = int(round((3 + (1 + 8 * K) ** 0.5) / 2))
+    assert (n - 1) * (n - 2) // 2 == K, "bad packed size"
+    return (c.shape[0] if layout == PACKED_ROW else c.shape[1]), n
+
+
 def opt(c: np.ndarray, return_table: bool = False):
     """Algorithm OPT on one dense n x n weight matrix.
     Returns M[1, n-1]; with return_table also the (n-1)x(n-1) table
@@ -171,10 +184,7 @@ def bulk_opt(c: np.ndarray, layout: int, nthreads: int = 1,
     c: [p, n, n] (ROW_WISE) or [n, n, p] (COLUMN_WISE); returns out[p]
     (entries outside [h0, h1) are 0)."""
     c = np.ascontiguousarray(c)
-    if layout == ROW_WISE:
-        p, n, _ = c.shape
-    else:
-        n, _, p = c.shape
+    p, n = _tri_pn(c, layout)
     h1 = p if h1 is None else h1
     out = np.zeros(p, dtype=c.dtype)
     rc = lib().oracle_bulk_opt(_ptr(c), _ptr(out), n, p, _DT[_dtname(c)], layout, h0, h1, nthreads)
@@ -209,10 +219,7 @@ def brute_opt_set(c: np.ndarray):
 def bulk_opt_chords(c: np.ndarray, layout: int):
     """Parallel Algorithm OPT with chords for every instance: (out[p], chords[p, n-3, 2])."""
     c = np.ascontiguousarray(c)
-    if layout == ROW_WISE:
-        p, n, _ = c.shape
-    else:
-        n, _, p = c.shape
+    p, n = _tri_pn(c, layout)
     out = np.zeros(p, dtype=c.dtype)
     ch = np.zeros((p, max(n - 3, 0), 2), dtype=np.int16)
     rc = lib().oracle_bulk_opt_chords(_ptr(c), _ptr(out), _ptr(ch), n, p, _DT[_dtname(c)], layout, 0, p)

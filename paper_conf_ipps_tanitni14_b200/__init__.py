@@ -21,7 +21,7 @@ import torch
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libbulkobl.so")
 
-ROW_WISE, COLUMN_WISE = 0, 1
+ROW_WISE, COLUMN_WISE, PACKED_ROW, PACKED_COLUMN = 0, 1, 2, 3
 I32, F32 = 0, 1
 AUTO = 0
 PS_ACROSS, PS_WARPSCAN, PS_FUSED_ROW, PS_TRANSPOSED, PS_NAIVE = 1, 2, 3, 4, 5
@@ -161,6 +161,14 @@ def prefix_sums_host(x_host: torch.Tensor, layout: int = ROW_WISE, variant: int 
 
 # ---------------------------------------------------------- triangulation
 def _tri_shape(c: torch.Tensor, layout: int):
+    if layout in (PACKED_ROW, PACKED_COLUMN):
+        if c.dim() != 2:
+            raise ValueError("packed weights are [p, K] (PACKED_ROW) or [K, p] (PACKED_COLUMN)")
+        K, p = (c.shape[1], c.shape[0]) if layout == PACKED_ROW else (c.shape[0], c.shape[1])
+        n = int(round((3 + (1 + 8 * K) ** 0.5) / 2))
+        if (n - 1) * (n - 2) // 2 != K:
+            raise ValueError("packed size K must be (n-1)(n-2)/2")
+        return n, p
     if c.dim() != 3:
         raise ValueError("weights are [p, n, n] (ROW_WISE) or [n, n, p] (COLUMN_WISE)")
     if layout == ROW_WISE:
@@ -241,7 +249,8 @@ def triangulation_host(c_host: torch.Tensor, layout: int = ROW_WISE, variant: in
     if out_host is None:
         out_host = torch.empty(p, dtype=c_host.dtype).pin_memory()
     if device_buf is None:
-        need = n * n * p * 4 + p * 4 + triangulation_workspace(n, p, dt, layout, variant)
+        words = (n - 1) * (n - 2) // 2 if layout in (PACKED_ROW, PACKED_COLUMN) else n * n
+        need = words * p * 4 + p * 4 + triangulation_workspace(n, p, dt, layout, variant)
         device_buf = torch.empty(need, dtype=torch.uint8, device="cuda")
     _check(lib().bulk_triangulation_host(c_host.data_ptr(), out_host.data_ptr(), n, p, dt, layout, variant,
                                          device_buf.data_ptr(), device_buf.numel(), _stream(stream)))
@@ -274,7 +283,8 @@ def generate_prefix(n: int, p: int, seed: int, dtype=torch.float32, layout: int 
 
 def generate_tri(n: int, p: int, seed: int, dtype=torch.float32, layout: int = ROW_WISE, h0: int = 0,
                  device="cuda", out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
-    shape = (p, n, n) if layout == ROW_WISE else (n, n, p)
+    K = (n - 1) * (n - 2) // 2
+    shape = {ROW_WISE: (p, n, n), COLUMN_WISE: (n, n, p), PACKED_ROW: (p, K), PACKED_COLUMN: (K, p)}[layout]
     if out is None:
         out = torch.empty(shape, dtype=dtype, device=device)
     _check(lib().bulk_generate_tri(out.data_ptr(), n, p, h0, seed, _dtype_code(out), layout, _stream(stream)))

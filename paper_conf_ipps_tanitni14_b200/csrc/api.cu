@@ -73,6 +73,9 @@ static constexpr int64_t kMaxElems = int64_t(1) << 40;
 
 static bool valid_dtype(int d) { return d == BO_I32 || d == BO_F32; }
 static bool valid_layout(int l) { return l == BO_ROW_WISE || l == BO_COLUMN_WISE; }
+static bool valid_tri_layout(int l) { return l >= BO_ROW_WISE && l <= BO_PACKED_COLUMN; }
+// weights per instance in a layout: n*n dense, (n-1)(n-2)/2 packed
+static int64_t tri_words(int64_t n, int layout) { return layout >= BO_PACKED_ROW ? (n - 1) * (n - 2) / 2 : n * n; }
 
 static bool ranges_partially_overlap(const void *a, const void *b, size_t bytes) {
     const uintptr_t x = reinterpret_cast<uintptr_t>(a), y = reinterpret_cast<uintptr_t>(b);
@@ -111,7 +114,7 @@ static int check_tri_args(const void *c, const void *out, int64_t n, int64_t p, 
     if (n < 3 || n > 4096) return fail(BO_EINVAL, "triangulation: need 3 <= n <= 4096");
     if (p < 0) return fail(BO_EINVAL, "triangulation: p must be >= 0");
     if (!valid_dtype(dtype)) return fail(BO_EINVAL, "triangulation: dtype must be BO_I32 or BO_F32");
-    if (!valid_layout(layout)) return fail(BO_EINVAL, "triangulation: bad layout");
+    if (!valid_tri_layout(layout)) return fail(BO_EINVAL, "triangulation: bad layout");
     if (p > kMaxElems / (n * n)) return fail(BO_EINVAL, "triangulation: n*n*p too large");
     if (p > 0 && (!c || !out)) return fail(BO_EINVAL, "triangulation: NULL pointer");
     if (variant != BO_AUTO && (variant < BO_TRI_UMM_GLOBAL || variant > BO_TRI_TILED_GLOBAL))
@@ -280,7 +283,8 @@ int bulk_generate_prefix(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t s
 int bulk_generate_tri(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout,
                       void *stream) {
     t_err.clear();
-    if (n < 1 || p < 0 || h0 < 0 || !valid_dtype(dtype) || !valid_layout(layout))
+    if (n < 1 || p < 0 || h0 < 0 || !valid_dtype(dtype) || !valid_tri_layout(layout) ||
+        (layout >= BO_PACKED_ROW && n < 3))
         return fail(BO_EINVAL, "generate_tri: bad argument");
     if (p > 0 && !dst) return fail(BO_EINVAL, "generate_tri: NULL pointer");
     return launch_gen_tri(dst, n, p, h0, seed, dtype, layout, static_cast<cudaStream_t>(stream));
@@ -356,7 +360,7 @@ int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, 
     if (p == 0) return BO_OK;
     const int v = resolve_tri_variant(n, p, dtype, layout, variant);
     const int64_t ch = host_chunk(p);
-    const size_t nn = static_cast<size_t>(n) * n;
+    const size_t nn = static_cast<size_t>(tri_words(n, layout));     // weights per instance
     const size_t c_bytes = nn * p * 4, out_bytes = static_cast<size_t>(p) * 4;
     const size_t ws_bytes = tri_workspace(n, p, v);
     if (!d_buf || d_bytes < c_bytes + out_bytes + ws_bytes)
@@ -377,7 +381,7 @@ int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, 
         const int64_t pc = std::min(ch, p - p0);
         cudaStream_t s = hp->s[k & 1];
         char *dchunk = db + static_cast<size_t>(p0) * nn * 4;
-        if (layout == BO_ROW_WISE)
+        if (layout == BO_ROW_WISE || layout == BO_PACKED_ROW)
             rc = cuda_check(cudaMemcpyAsync(dchunk, hc + static_cast<size_t>(p0) * nn * 4, pc * nn * 4,
                                             cudaMemcpyHostToDevice, s),
                             "tri_host: H2D");

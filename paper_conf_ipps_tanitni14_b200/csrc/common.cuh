@@ -155,6 +155,21 @@ __device__ __forceinline__ uint32_t swz128(uint32_t row, uint32_t chunk) {
     return row * 128u + ((chunk ^ (row & 7u)) << 4);
 }
 
+// ---------------------------------------------------------------- weights
+// Index of the chord weight c[a][b] of instance h in the four weight layouts
+// (include/bulkobl.h): dense row-wise c[h*n*n + a*n + b], dense column-wise
+// c[(a*n + b)*p + h], packed (b - a >= 2 only, K = (n-1)(n-2)/2 per instance,
+// k = a(n-2) - a(a-1)/2 + (b-a-2)) row-wise c[h*K + k] or column-wise c[k*p + h].
+__host__ __device__ __forceinline__ long long tri_c_index(int layout, long long h, long long n, long long p,
+                                                          long long a, long long b) {
+    if (layout <= BO_COLUMN_WISE) {
+        const long long e = a * n + b;
+        return layout == BO_ROW_WISE ? h * n * n + e : e * p + h;
+    }
+    const long long K = (n - 1) * (n - 2) / 2, k = a * (n - 2) - a * (a - 1) / 2 + (b - a - 2);
+    return layout == BO_PACKED_ROW ? h * K + k : k * p + h;
+}
+
 // ---------------------------------------------------------------- arithmetic
 // int32 adds wrap mod 2^32 (two's complement), done in uint32 to avoid UB.
 __device__ __forceinline__ int32_t add_wrap(int32_t a, int32_t b) {

@@ -50,20 +50,22 @@ __global__ void gen_prefix_kernel(uint32_t *dst, long long n, long long p, long 
 
 __global__ void gen_tri_kernel(uint32_t *dst, long long n, long long p, long long h0, uint64_t seed, int dtype,
                                int layout) {
+    // walks the dense (h, a, b) space; packed layouts store only b - a >= 2
     const long long nn = n * n, total = nn * p;
     for (long long idx = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; idx < total;
          idx += static_cast<long long>(gridDim.x) * blockDim.x) {
         long long h, e;
-        if (layout == BO_ROW_WISE) { h = idx / nn; e = idx - h * nn; }
-        else { e = idx / p; h = idx - e * p; }
+        if (layout == BO_COLUMN_WISE) { e = idx / p; h = idx - e * p; }
+        else { h = idx / nn; e = idx - h * nn; }
         const long long a = e / n, b = e - a * n;
+        if (layout >= BO_PACKED_ROW && b - a < 2) continue;
         uint32_t bits = 0;
         if (b - a >= 2 && !(a == 0 && b == n - 1)) {
             const uint64_t u = gen_u(seed, static_cast<uint64_t>(h0 + h), static_cast<uint64_t>(e));
             bits = dtype == BO_I32 ? static_cast<uint32_t>(u >> 44)
                                    : __float_as_uint(static_cast<float>(u >> 40) * 0x1p-24f);
         }
-        dst[idx] = bits;
+        dst[layout >= BO_PACKED_ROW ? tri_c_index(layout, h, n, p, a, b) : idx] = bits;
     }
 }
 

@@ -50,8 +50,7 @@ struct MinPlus<float> {
 
 __host__ __device__ __forceinline__ long long c_index(int layout, long long h, long long n, long long p,
                                                       long long a, long long b) {
-    const long long e = a * n + b;
-    return layout == BO_ROW_WISE ? h * n * n + e : e * p + h;
+    return tri_c_index(layout, h, n, p, a, b);
 }
 
 // -------------------------------------------------------------- THREAD_REG
@@ -89,7 +88,8 @@ template <typename T, int N, int LAYOUT>
 __global__ void __launch_bounds__(32)
 tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out, long long p, long long nbatch) {
     using Op = MinPlus<T>;
-    constexpr int NE = (N - 3) * N + N;          // c[N-3][N-1] is the last weight read
+    constexpr int NE = LAYOUT == BO_PACKED_ROW ? (N - 1) * (N - 2) / 2   // packed: every weight is read
+                                               : (N - 3) * N + N;        // c[N-3][N-1] is the last one read
     constexpr int NB = (NE + 31) / 32;
     constexpr uint32_t kBatchBytes = NB * 4096;
     extern __shared__ uint8_t smem_raw[];
@@ -102,7 +102,7 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
         mbar_arrive_expect_tx(&bar[i & 1], kBatchBytes);
 #pragma unroll
         for (int k = 0; k < NB; ++k) {
-            if (LAYOUT == BO_ROW_WISE) tma_load_2d(dst + k * 4096, &cmap, k * 32, static_cast<int>(b * 32), &bar[i & 1]);
+            if (LAYOUT != BO_COLUMN_WISE) tma_load_2d(dst + k * 4096, &cmap, k * 32, static_cast<int>(b * 32), &bar[i & 1]);
             else tma_load_2d(dst + k * 4096, &cmap, static_cast<int>(b * 32), k * 32, &bar[i & 1]);
         }
     };
@@ -120,9 +120,13 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
         if (t == 0 && b + gridDim.x < nbatch) issue(i + 1);   // the other buffer was released last iteration
         mbar_wait(&bar[i & 1], static_cast<uint32_t>((i >> 1) & 1));
         const uint8_t *cur = buf + (i & 1) * kBatchBytes;
-        auto cl = [&](int e) -> T {
+        auto cl = [&](int e) -> T {                 // e = dense index a*N + b (compile time)
+            if (LAYOUT == BO_PACKED_ROW) {
+                const int a = e / N, b = e % N;
+                e = a * (N - 2) - a * (a - 1) / 2 + (b - a - 2);
+            }
             const uint8_t *box = cur + (e >> 5) * 4096;
-            if (LAYOUT == BO_ROW_WISE) {
+            if (LAYOUT != BO_COLUMN_WISE) {
                 const uint4 v = *reinterpret_cast<const uint4 *>(box + swz128(t, (e & 31) >> 2));
                 const uint32_t w = (e & 3) == 0 ? v.x : (e & 3) == 1 ? v.y : (e & 3) == 2 ? v.z : v.w;
                 return *reinterpret_cast<const T *>(&w);
@@ -145,6 +149,76 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
         const long long h = b * 32 + t;
         if (h < p) out[h] = M[1][N - 1];
         __syncwarp();                                        // buffer i&1 free for batch i+2
+    }
+}
+
+
+// THREAD_REG on packed row-wise weights (NEXT-4): a batch of 32 consecutive
+// instances is one contiguous run of 32*K words, moved by a single 1-D bulk
+// copy (cp.async.bulk) into shared memory; thread t reads its instance's
+// weights at t*K + k (K odd for every n = 0,1 mod 4... and any odd stride is
+// bank-conflict-free).  Persistent CTAs, two buffers: the next batch streams
+// in while the current one computes.  A ragged last batch reads global memory.
+__device__ __forceinline__ void bulk_load_1d(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+
+template <typename T, int N>
+__global__ void __launch_bounds__(32)
+tri_thread_reg_packed(const T *__restrict__ c, T *__restrict__ out, long long p, long long nbatch) {
+    using Op = MinPlus<T>;
+    constexpr int K = (N - 1) * (N - 2) / 2;
+    constexpr uint32_t kBatchBytes = 32u * K * sizeof(T);
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 127) & ~uintptr_t(127));
+    uint64_t *bar = reinterpret_cast<uint64_t *>(buf + 2 * ((kBatchBytes + 127) & ~127u));
+    const uint32_t stride = (kBatchBytes + 127) & ~127u;
+    const int t = threadIdx.x;
+    const long long nfull = p / 32;                      // batches that are complete
+    auto issue = [&](long long i) {
+        const long long b = blockIdx.x + i * gridDim.x;
+        if (b >= nfull) return;
+        mbar_arrive_expect_tx(&bar[i & 1], kBatchBytes);
+        bulk_load_1d(buf + (i & 1) * stride, c + b * 32 * K, kBatchBytes, &bar[i & 1]);
+    };
+    if (t == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        fence_barrier_init();
+        issue(0);
+    }
+    __syncwarp();
+    for (long long i = 0;; ++i) {
+        const long long b = blockIdx.x + i * gridDim.x;
+        if (b >= nbatch) break;
+        if (t == 0) issue(i + 1);
+        const bool full = b < nfull;
+        if (full) mbar_wait(&bar[i & 1], static_cast<uint32_t>((i >> 1) & 1));
+        const T *cur = reinterpret_cast<const T *>(buf + (i & 1) * stride) + t * K;
+        const long long h = b * 32 + t;
+        const T *g = c + (h < p ? h : 0) * K;
+        auto cl = [&](int a, int bb) -> T {
+            const int k = a * (N - 2) - a * (a - 1) / 2 + (bb - a - 2);
+            return full ? cur[k] : __ldg(g + k);
+        };
+        T M[N][N];
+#pragma unroll
+        for (int ii = 1; ii <= N - 1; ++ii) M[ii][ii] = T(0);
+#pragma unroll
+        for (int ii = N - 2; ii >= 1; --ii) {
+#pragma unroll
+            for (int j = ii + 1; j <= N - 1; ++j) {
+                T s = Op::inf();
+#pragma unroll
+                for (int k = ii; k <= j - 1; ++k) s = Op::addmin(M[ii][k], M[k + 1][j], s);
+                M[ii][j] = Op::add(s, cl(ii - 1, j));
+            }
+        }
+        if (h < p) out[h] = M[1][N - 1];
+        __syncwarp();
     }
 }
 
@@ -188,12 +262,11 @@ tri_smem_warp(const T *__restrict__ c, T *__restrict__ out, int n, long long p, 
 
     for (long long hb = static_cast<long long>(blockIdx.x) * W; hb < p; hb += static_cast<long long>(gridDim.x) * W) {
         const long long h = hb + warp;
-        if (layout == BO_ROW_WISE) {
+        if (layout != BO_COLUMN_WISE) {
             if (h < p) {
-                const T *ch = c + h * n * n;
                 for (int a = 0; a < n1; ++a)
                     for (int b = a + lane; b < n1; b += 32)
-                        S[a * SP + b] = b == a ? T(0) : __ldg(ch + a * n + b + 1);
+                        S[a * SP + b] = b == a ? T(0) : __ldg(c + c_index(layout, h, n, p, a, b + 1));
             }
         } else {
             // column-wise c[(a*n+b)*p + h]: consecutive threads take consecutive
@@ -270,9 +343,10 @@ static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) 
     constexpr int NB = (NE + 31) / 32;
     constexpr size_t smem = 1024 + 2 * NB * 4096 + 16;
     CUtensorMap map;
-    const bool ok = LAYOUT == BO_ROW_WISE
-                        ? make_tmap_2d(&map, c, p, N * N, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
-                        : make_tmap_2d(&map, c, N * N, p, 32, 32, CU_TENSOR_MAP_SWIZZLE_NONE);
+    constexpr int K = (N - 1) * (N - 2) / 2;
+    const bool ok = LAYOUT == BO_ROW_WISE     ? make_tmap_2d(&map, c, p, N * N, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
+                    : LAYOUT == BO_PACKED_ROW ? make_tmap_2d(&map, c, p, K, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
+                                              : make_tmap_2d(&map, c, N * N, p, 32, 32, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (!ok) return fail(BO_ECUDA, "triangulation THREAD_REG: cuTensorMapEncodeTiled failed");
     static bool attr = [] {
         return cudaFuncSetAttribute(tri_thread_reg_tma<T, N, LAYOUT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -289,7 +363,27 @@ static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) 
 }
 
 template <typename T, int N>
+static int launch_reg_packed(const void *c, void *out, int64_t p, cudaStream_t st) {
+    constexpr int K = (N - 1) * (N - 2) / 2;
+    constexpr size_t batch = (32u * K * sizeof(T) + 127) & ~size_t(127);
+    constexpr size_t smem = 128 + 2 * batch + 16;
+    static bool attr = [] {
+        return cudaFuncSetAttribute(tri_thread_reg_packed<T, N>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    static_cast<int>(smem)) == cudaSuccess;
+    }();
+    if (!attr) return fail(BO_ECUDA, "triangulation THREAD_REG packed: cannot set dynamic smem");
+    const long long nbatch = (p + 31) / 32;
+    int per_sm = 1;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_thread_reg_packed<T, N>, 32, smem);
+    const long long grid = std::min<long long>(nbatch, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
+    tri_thread_reg_packed<T, N><<<static_cast<unsigned>(grid), 32, smem, st>>>(
+        static_cast<const T *>(c), static_cast<T *>(out), p, nbatch);
+    return after_launch("tri_thread_reg_packed");
+}
+
+template <typename T, int N>
 static int launch_reg_n(const void *c, void *out, int64_t p, int layout, cudaStream_t st) {
+    if (layout == BO_PACKED_ROW && N >= 4 && aligned16(c)) return launch_reg_packed<T, N>(c, out, p, st);
     if (p >= 32 && N >= 6 && p < (int64_t(1) << 31) && aligned16(c)) {
         if (layout == BO_ROW_WISE && (N * N) % 4 == 0) return launch_reg_tma<T, N, BO_ROW_WISE>(c, out, p, st);
         // column-wise c is already coalesced for thread-per-instance: direct loads win (measured 14.5 vs 19.3 us)

@@ -188,15 +188,16 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
                 }
             }
             tt::cp_async_wait_all();
-        } else if (layout == BO_COLUMN_WISE) {
-            // Column-wise weights c[(a*n+b)*p + h]: the whole CTA loads the
+        } else if (layout == BO_COLUMN_WISE || layout == BO_PACKED_COLUMN) {
+            // Column-wise weights c[(a*n+b)*p + h] or packed c[k*p + h]: the whole CTA loads the
             // weights of its `ninst` consecutive instances together, instance index
             // fastest, so each warp request covers whole 32-byte sectors.
             __syncthreads();                                // every table of the CTA is free
             T *Z0 = reinterpret_cast<T *>(smem_raw);
             for (int a = 0; a < n - 2; ++a) {
                 const int L = n - a - 2;                    // cells (a, a+2 .. n-1)
-                const long long row0 = static_cast<long long>(a) * n + a + 2;
+                const long long row0 = layout == BO_COLUMN_WISE ? static_cast<long long>(a) * n + a + 2
+                                                                : tri_c_index(BO_PACKED_COLUMN, 0, n, 1, a, a + 2);
                 for (int idx = threadIdx.x; idx < L * ninst; idx += blockDim.x) {
                     const int q = idx % ninst, b = a + 2 + idx / ninst;
                     if (base + q < p)
@@ -207,8 +208,11 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             tt::cp_async_wait_all();
             __syncthreads();
         } else if (live) {
+            // packed row-wise or unaligned dense row-wise: 4-byte asynchronous copies
+            // (a packed row is contiguous, so lanes read consecutive words)
             for (int a = 0; a < n - 2; ++a)
-                for (int b = a + 2 + li; b < n; b += LPI) Z[tt::xoff(a, b)] = __ldg(c + h * nn + static_cast<long long>(a) * n + b);
+                for (int b = a + 2 + li; b < n; b += LPI) tt::cp_async4(Z + tt::xoff(a, b), c + tri_c_index(layout, h, n, p, a, b));
+            tt::cp_async_wait_all();
         }
         __syncwarp();
 
@@ -450,10 +454,7 @@ tri_tiled_global_kernel(const T *__restrict__ c, T *__restrict__ out, T *ws, int
             }
         } else {
             for (int a = 0; a < n - 2; ++a)
-                for (int b = a + 2 + tid; b < n; b += nthr) {
-                    const long long e = static_cast<long long>(a) * n + b;
-                    Z[tt::xoff(a, b)] = __ldg(c + (layout == BO_ROW_WISE ? h * nn + e : e * p + h));
-                }
+                for (int b = a + 2 + tid; b < n; b += nthr) Z[tt::xoff(a, b)] = __ldg(c + tri_c_index(layout, h, n, p, a, b));
         }
         __syncthreads();
         // 2. D = 0

@@ -50,7 +50,7 @@ def test_device_generator_equals_bulkgen(dt, layout, kind):
 
 
 @pytest.mark.parametrize("dt", ["int32", "float32"])
-@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE, bo.PACKED_ROW, bo.PACKED_COLUMN])
 def test_device_tri_generator_equals_bulkgen(dt, layout):
     n, p, h0 = 13, 29, 5
     got = bo.generate_tri(n, p, 3, getattr(torch, dt), layout, h0=h0).cpu().numpy()
@@ -86,7 +86,7 @@ def test_prefix_host_transposed_variant():
     assert np.array_equal(out.numpy().view(np.uint32), oracle.bulk_prefix_sums(x, 0).view(np.uint32))
 
 
-@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE, bo.PACKED_ROW, bo.PACKED_COLUMN])
 @pytest.mark.parametrize("variant", [bo.AUTO, bo.TRI_UMM_GLOBAL])
 def test_tri_host_entry_point(layout, variant):
     n, p = 16, 2000

@@ -27,6 +27,8 @@ def _variants(n):
 
 
 def _supported(n, variant):
+    if variant in (bo.TRI_TILED, bo.TRI_TILED_HALF) and n > 64:
+        return False
     if variant in (bo.TRI_TILED, bo.TRI_TILED_HALF):
         try:
             bo.triangulation(torch.zeros((1, n, n), device=DEV), bo.ROW_WISE, bo.TRI_TILED)
@@ -41,8 +43,11 @@ CASES = [(3, 5), (4, 33), (5, 64), (8, 100), (13, 257), (16, 300), (17, 64), (18
          (40, 70), (63, 33), (64, 130), (65, 20), (100, 9), (128, 4)]
 
 
+LAYOUTS = [bo.ROW_WISE, bo.COLUMN_WISE, bo.PACKED_ROW, bo.PACKED_COLUMN]
+
+
 @pytest.mark.parametrize("dt", ["int32", "float32"])
-@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("layout", LAYOUTS)
 @pytest.mark.parametrize("n,p", CASES)
 def test_all_variants_match_oracle(dt, layout, n, p):
     c = bulkgen.tri_input(n, p, seed=n + 100 * p, dtype=dt, layout=layout)
@@ -79,7 +84,7 @@ def test_hand_worked_pentagon():
     assert got.tolist() == [7]      # tests/golden/pentagon_worked.txt
 
 
-@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("layout", LAYOUTS)
 def test_tr1_full_config(layout):
     n, p = 16, 65536
     c = bo.generate_tri(n, p, 3, torch.int32, layout)
@@ -115,7 +120,7 @@ def test_tr2_variants_agree_full_size(variant):
 
 # ------------------------------------------------------------------ NEXT-1 chords
 @pytest.mark.parametrize("dt", ["int32", "float32"])
-@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("layout", LAYOUTS)
 @pytest.mark.parametrize("n,p", [(3, 7), (4, 40), (5, 33), (8, 100), (13, 64), (16, 300), (17, 50), (33, 64),
                                  (61, 20), (64, 130)])
 def test_chords_match_oracle(dt, layout, n, p):

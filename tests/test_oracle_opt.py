@@ -230,3 +230,29 @@ def test_bulk_chords_layouts_agree():
     for h in range(p):
         v, ch = oracle.opt_chords(row[h])
         assert v == a[h] and np.array_equal(ch, ca[h])
+
+
+# ------------------------------------------------- NEXT-4: packed weight layouts
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("n", [3, 4, 7, 16])
+def test_packed_layouts_give_the_dense_results(dt, n):
+    p = 13
+    dense = bulkgen.tri_input(n, p, seed=n, dtype=dt)
+    ref = oracle.bulk_opt(dense, oracle.ROW_WISE)
+    for layout in (oracle.PACKED_ROW, oracle.PACKED_COLUMN):
+        pk = bulkgen.tri_input(n, p, seed=n, dtype=dt, layout=layout)
+        K = (n - 1) * (n - 2) // 2
+        assert pk.shape == ((p, K) if layout == oracle.PACKED_ROW else (K, p))
+        assert np.array_equal(oracle.bulk_opt(pk, layout).view(np.uint32), ref.view(np.uint32))
+        v, ch = oracle.bulk_opt_chords(pk, layout)
+        assert np.array_equal(ch, oracle.bulk_opt_chords(dense, oracle.ROW_WISE)[1])
+
+
+def test_packed_index_closed_form():
+    n = 9
+    pairs = bulkgen.packed_pairs(n)
+    assert len(pairs) == (n - 1) * (n - 2) // 2
+    for k, (a, b) in enumerate(pairs):
+        assert k == a * (n - 2) - a * (a - 1) // 2 + (b - a - 2)
+    # every weight Algorithm OPT reads appears exactly once (trace test: {b-a >= 2})
+    assert sorted(pairs) == sorted((a, b) for a in range(n) for b in range(a + 2, n))
