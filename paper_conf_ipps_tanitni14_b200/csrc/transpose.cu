@@ -14,7 +14,10 @@ namespace bo {
 namespace tr {
 constexpr int kCols = 32;                      // box inner extent (128 B)
 constexpr int kRows = 64;                      // box outer extent (2 sub-tiles)
-constexpr int kStages = 6;
+#ifndef BO_TR_STAGES
+#define BO_TR_STAGES 6
+#endif
+constexpr int kStages = BO_TR_STAGES;
 constexpr int kOut = 2;
 constexpr int kThreads = 256;
 constexpr uint32_t kBoxBytes = kRows * kCols * 4;   // 8 KiB
