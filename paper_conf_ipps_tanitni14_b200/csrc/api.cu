@@ -5,7 +5,9 @@
 
 #include <cstring>
 #include <mutex>
+#include <set>
 #include <string>
+#include <utility>
 #include <vector>
 
 namespace bo {
@@ -22,6 +24,19 @@ int fail(int status, const std::string &msg) {
 int cuda_check(cudaError_t e, const char *what) {
     if (e == cudaSuccess) return BO_OK;
     return fail(BO_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+
+bool ensure_dyn_smem(const void *func, int bytes) {
+    static std::mutex mu;
+    static std::set<std::pair<int, std::pair<const void *, int>>> done;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return false;
+    const auto key = std::make_pair(dev, std::make_pair(func, bytes));
+    std::lock_guard<std::mutex> g(mu);
+    if (done.count(key)) return true;
+    if (cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess) return false;
+    done.insert(key);
+    return true;
 }
 
 // ---------------------------------------------------------------- TMA maps
@@ -150,9 +165,13 @@ static HostPipe *host_pipe() {
     return pipes[dev];
 }
 
+#ifndef BO_HOST_CHUNKS
+#define BO_HOST_CHUNKS 32     // measured: 8 -> 95.2 ms, 32 -> 89.8 ms per 8 GiB round trip (PCIe-bound)
+#endif
 static int64_t host_chunk(int64_t p) {
-    // ~8 chunks, multiple of 128 instances, so copies of chunk k+1 overlap compute/copy-back of chunk k
-    int64_t ch = (p + 7) / 8;
+    // BO_HOST_CHUNKS chunks, multiple of 128 instances, so copies of chunk k+1
+    // overlap compute/copy-back of chunk k
+    int64_t ch = (p + BO_HOST_CHUNKS - 1) / BO_HOST_CHUNKS;
     ch = ((ch + 127) / 128) * 128;
     return std::max<int64_t>(std::min<int64_t>(ch, p), 1);
 }

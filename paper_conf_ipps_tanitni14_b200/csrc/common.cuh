@@ -28,6 +28,10 @@ inline int after_launch(const char *what) {
     return cuda_check(cudaGetLastError(), what);
 }
 
+// Opt a kernel into `bytes` of dynamic shared memory on the current device;
+// done once per (device, kernel) -- processes may drive several GPUs.
+bool ensure_dyn_smem(const void *func, int bytes);
+
 inline int num_sms() {
     static int sms = [] {
         int dev = 0, v = 148;

@@ -329,10 +329,7 @@ static int launch_fused_row_tma(const T *src, T *dst, int64_t n, int64_t p, cuda
     if (!make_tmap_2d(&smap, src, p, n, INST, fr::kElems, CU_TENSOR_MAP_SWIZZLE_128B) ||
         !make_tmap_2d(&dmap, dst, p, n, INST, fr::kElems, CU_TENSOR_MAP_SWIZZLE_128B))
         return fail(BO_ECUDA, "prefix fused-row: cuTensorMapEncodeTiled failed");
-    static bool attr = [] {
-        return cudaFuncSetAttribute(ps_fused_row_tma<T, INST>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    static_cast<int>(C::kSmem)) == cudaSuccess;
-    }();
+    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&ps_fused_row_tma<T, INST>), static_cast<int>(C::kSmem));
     if (!attr) return fail(BO_ECUDA, "prefix fused-row: cannot set dynamic smem");
     const long long ntiles = (p + INST - 1) / INST;
     const int nchunks = static_cast<int>((n + fr::kElems - 1) / fr::kElems);

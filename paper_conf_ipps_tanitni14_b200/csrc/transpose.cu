@@ -142,10 +142,7 @@ int launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, cud
         if (!make_tmap_2d(&smap, src, rows, cols, tr::kRows, tr::kCols, CU_TENSOR_MAP_SWIZZLE_128B) ||
             !make_tmap_2d(&dmap, dst, cols, rows, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B))
             return fail(BO_ECUDA, "transpose: cuTensorMapEncodeTiled failed");
-        static bool attr = [] {
-            return cudaFuncSetAttribute(transpose_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        static_cast<int>(tr::kSmem)) == cudaSuccess;
-        }();
+        const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&transpose_tma_kernel), static_cast<int>(tr::kSmem));
         if (!attr) return fail(BO_ECUDA, "transpose: cannot set dynamic smem");
         const long long tiles_c = (cols + tr::kCols - 1) / tr::kCols;
         const long long tiles_r = (rows + tr::kRows - 1) / tr::kRows;

@@ -349,10 +349,7 @@ static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) 
                     : LAYOUT == BO_PACKED_ROW ? make_tmap_2d(&map, c, p, K, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
                                               : make_tmap_2d(&map, c, N * N, p, 32, 32, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (!ok) return fail(BO_ECUDA, "triangulation THREAD_REG: cuTensorMapEncodeTiled failed");
-    static bool attr = [] {
-        return cudaFuncSetAttribute(tri_thread_reg_tma<T, N, LAYOUT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    static_cast<int>(smem)) == cudaSuccess;
-    }();
+    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_thread_reg_tma<T, N, LAYOUT>), static_cast<int>(smem));
     if (!attr) return fail(BO_ECUDA, "triangulation THREAD_REG: cannot set dynamic smem");
     const long long nbatch = (p + 31) / 32;
     int per_sm = 1;
@@ -368,10 +365,7 @@ static int launch_reg_packed(const void *c, void *out, int64_t p, cudaStream_t s
     constexpr int K = (N - 1) * (N - 2) / 2;
     constexpr size_t batch = (32u * K * sizeof(T) + 127) & ~size_t(127);
     constexpr size_t smem = 128 + 2 * batch + 16;
-    static bool attr = [] {
-        return cudaFuncSetAttribute(tri_thread_reg_packed<T, N>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    static_cast<int>(smem)) == cudaSuccess;
-    }();
+    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_thread_reg_packed<T, N>), static_cast<int>(smem));
     if (!attr) return fail(BO_ECUDA, "triangulation THREAD_REG packed: cannot set dynamic smem");
     const long long nbatch = (p + 31) / 32;
     int per_sm = 1;
@@ -419,10 +413,7 @@ template <typename T>
 static int launch_smem_warp(const void *c, void *out, int64_t n, int64_t p, int layout, cudaStream_t st) {
     const size_t per = smem_per_instance(n);
     if (per > 200 * 1024) return fail(BO_EUNSUPPORTED, "triangulation SMEM_WARP: table does not fit in smem");
-    static bool attr = [] {
-        return cudaFuncSetAttribute(tri_smem_warp<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024) ==
-               cudaSuccess;
-    }();
+    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_smem_warp<T>), 227 * 1024);
     if (!attr) return fail(BO_ECUDA, "triangulation SMEM_WARP: cannot set dynamic smem");
     // warps per CTA: as many instances as fit in one SM's smem, at most 16
     int W = static_cast<int>(std::min<size_t>(16, (227 * 1024) / per));

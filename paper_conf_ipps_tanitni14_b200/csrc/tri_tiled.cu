@@ -384,10 +384,7 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
         if (resident > best || (layout == BO_COLUMN_WISE && resident == best)) best = resident, W = w;
     }
     const size_t smem = W * IPW * per_inst;
-    static bool attr = [] {
-        return cudaFuncSetAttribute(tri_tiled_kernel<T, LPI, CHORDS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    227 * 1024) == cudaSuccess;
-    }();
+    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_tiled_kernel<T, LPI, CHORDS>), 227 * 1024);
     if (!attr) return fail(BO_ECUDA, "tiled: cannot set dynamic smem");
     int per_sm = 1;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_tiled_kernel<T, LPI, CHORDS>, W * 32, smem);
