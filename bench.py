@@ -186,15 +186,22 @@ class ClockSampler:
 
 
 class Ctx:
-    def __init__(self):
+    def __init__(self, backend="nccl"):
         self.rank = int(os.environ.get("RANK", 0))
         self.world = int(os.environ.get("WORLD_SIZE", 1))
         self.local = int(os.environ.get("LOCAL_RANK", 0))
         self.dist = self.world > 1
+        self.backend = backend
+        # one process per GPU; the modulo only matters for the gloo test mode
+        # (several ranks sharing one GPU to exercise the multi-rank logic)
+        self.device = self.local % max(1, torch.cuda.device_count()) if torch.cuda.is_available() else 0
 
     def barrier(self):
         if self.dist:
-            dist.barrier(device_ids=[self.local])
+            if self.backend == "nccl":
+                dist.barrier(device_ids=[self.device])
+            else:
+                dist.barrier()
 
     def max(self, x: float) -> float:
         from paper_conf_ipps_tanitni14_b200 import shard
@@ -445,7 +452,7 @@ def run_ours(args, ctx):
     traffic = load_traffic()
     stream = torch.cuda.Stream()
     name = args.workload
-    sampler = ClockSampler(torch.cuda.current_device() if not ctx.dist else ctx.local)
+    sampler = ClockSampler(ctx.device)
     # primary, with clocks sampled during its timed region
     wl = WORKLOADS[name]
     st = setup_workload(wl, ctx.rank)
@@ -579,21 +586,26 @@ def main():
     ap.add_argument("--no-extras", dest="extras", action="store_false")
     ap.add_argument("--no-e2e", dest="e2e", action="store_false")
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo only to test the multi-rank logic with several ranks on one GPU")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
-    ctx = Ctx()
+    ctx = Ctx(args.dist_backend)
     if args.impl == "reference":
         run_reference(args, ctx)
         return
-    torch.cuda.set_device(ctx.local)
+    torch.cuda.set_device(ctx.device)
     if ctx.dist:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", ctx.local))
+        if ctx.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", ctx.device))
+        else:
+            dist.init_process_group(ctx.backend)
     try:
         run_ours(args, ctx)
     finally:
         if ctx.dist:
-            dist.barrier(device_ids=[ctx.local])
+            ctx.barrier()
             dist.destroy_process_group()
 
 
