@@ -456,8 +456,15 @@ def run_ours(args, ctx):
     # primary, with clocks sampled during its timed region
     wl = WORKLOADS[name]
     st = setup_workload(wl, ctx.rank)
+    flush, l2note = None, f"input {input_bytes(wl) / 2 ** 30:.2f} GiB per GPU > 2x the 126 MB L2; no flush needed"
+    if input_bytes(wl) < 2 * L2_BYTES:
+        scratch = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device="cuda")
+        l2note = "input smaller than 2x L2: a 252 MB buffer is written between steps (outside the per-step events)"
+
+        def flush():
+            scratch.fill_(1)
     with sampler:
-        ms, launches = timed(ctx, st["fn"], args.steps, args.warmup, stream)
+        ms, launches = timed(ctx, st["fn"], args.steps, args.warmup, stream, flush)
     p_all = wl["p"] * ctx.world
     value = p_all / (ms * 1e-3)
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ctx.world, "steps": args.steps,
@@ -466,7 +473,7 @@ def run_ours(args, ctx):
             "config": {"workload": wl["desc"], "n": wl["n"], "p_per_gpu": wl["p"], "p_total": p_all,
                        "layout_in_out": "row-wise" if wl["layout"] == 0 else "column-wise",
                        "variant": st["variant"], "parallelism": f"instances sharded over {ctx.world} GPU(s)",
-                       "l2": "input 4 GiB per GPU > 126 MB L2; no flush needed",
+                       "l2": l2note,
                        "input": "counter-based synthetic, generated on device from global instance ids"},
             "gpu_launches": launches}
     # roofline of the dominant kernel (the only kernel of the step for AUTO)
