@@ -138,3 +138,20 @@ def test_ps1_full_config_exact():
             xi = x if layout == bo.ROW_WISE else np.ascontiguousarray(x.T)
             got = bo.prefix_sums(torch.from_numpy(xi).to(DEV), layout).cpu().numpy()
             assert np.array_equal(got, oracle.bulk_prefix_sums(xi, layout))
+
+
+def test_max_size_64bit_indexing():
+    # n*p = 2^32 elements (16 GiB in, 16 GiB out): every index past 2^31 must be 64-bit
+    n, p, seed = 1024, 2 ** 22, 11
+    x = bo.generate_prefix(n, p, seed, torch.float32, bo.ROW_WISE)
+    y = bo.prefix_sums(x, bo.ROW_WISE)
+    ids = np.array([0, 2 ** 21 - 1, 2 ** 21, 2 ** 22 - 129, p - 1])
+    got = y[torch.from_numpy(ids).to(DEV)].cpu().numpy()
+    ref = oracle.bulk_prefix_sums(bulkgen.prefix_instances(n, ids, seed, "float32"), oracle.ROW_WISE)
+    assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+    del y
+    xc = bo.transpose(x)
+    del x
+    yc = bo.prefix_sums(xc, bo.COLUMN_WISE)
+    got = yc[:, torch.from_numpy(ids).to(DEV)].T.contiguous().cpu().numpy()
+    assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))

@@ -173,3 +173,13 @@ def test_512gon_paper_config_sampled():
     ids = np.array([0, 511, 1023])
     ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 7, "float32"), oracle.ROW_WISE, nthreads=NTHREADS)
     assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32))
+
+
+def test_tr2_large_p_64bit_indexing():
+    # p = 2^21 instances of dense 64x64 weights = 32 GiB: instance offsets past 2^31 words
+    n, p, seed = 64, 2 ** 21, 12
+    c = bo.generate_tri(n, p, seed, torch.float32, bo.ROW_WISE)
+    got = bo.triangulation(c).cpu().numpy()
+    ids = np.array([0, 2 ** 19 + 3, 2 ** 20 + 7, p - 1])
+    ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, seed, "float32"), oracle.ROW_WISE, nthreads=NTHREADS)
+    assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32))
