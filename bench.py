@@ -405,17 +405,26 @@ def e2e(ctx, name, steps, warmup):
     wl = WORKLOADS[name]
     n, p = wl["n"], wl["p"]
     dt = getattr(torch, wl["dtype"])
-    if wl["algo"] != "prefix":
+    if wl["algo"] not in ("prefix", "tri"):
         return None
-    shape = (p, n) if wl["layout"] == 0 else (n, p)
+    tri = wl["algo"] == "tri"
+    dcode = bo.F32 if wl["dtype"] == "float32" else bo.I32
     err = None
     try:
-        dev = bo.generate_prefix(n, p, wl["seed"], dt, wl["layout"], "uniform", h0=ctx.rank * p)
-        h_in = torch.empty(shape, dtype=dt, pin_memory=True)
+        if tri:
+            dev = bo.generate_tri(n, p, wl["seed"], dt, wl["layout"], h0=ctx.rank * p)
+            in_bytes, out_bytes = dev.numel() * 4, p * 4
+            need = bo.triangulation_host_bytes(n, p, dcode, wl["layout"], wl["variant"])
+            h_out = torch.empty(p, dtype=dt, pin_memory=True)
+        else:
+            dev = bo.generate_prefix(n, p, wl["seed"], dt, wl["layout"], "uniform", h0=ctx.rank * p)
+            in_bytes = out_bytes = n * p * 4
+            need = bo.prefix_sums_host_bytes(n, p, dcode, wl["layout"], wl["variant"])
+            h_out = torch.empty(dev.shape, dtype=dt, pin_memory=True)
+        h_in = torch.empty(dev.shape, dtype=dt, pin_memory=True)
         h_in.copy_(dev)
-        h_out = torch.empty(shape, dtype=dt, pin_memory=True)
         del dev
-        dbuf = torch.empty(n * p * 4, dtype=torch.uint8, device="cuda")
+        dbuf = torch.empty(need, dtype=torch.uint8, device="cuda")
         torch.cuda.synchronize()
     except Exception as exc:        # agree across ranks before any barrier
         err = repr(exc)
@@ -424,7 +433,10 @@ def e2e(ctx, name, steps, warmup):
     stream = torch.cuda.current_stream()
 
     def fn():
-        bo.prefix_sums_host(h_in, wl["layout"], wl["variant"], out_host=h_out, device_buf=dbuf, stream=stream)
+        if tri:
+            bo.triangulation_host(h_in, wl["layout"], wl["variant"], out_host=h_out, device_buf=dbuf, stream=stream)
+        else:
+            bo.prefix_sums_host(h_in, wl["layout"], wl["variant"], out_host=h_out, device_buf=dbuf, stream=stream)
     for _ in range(warmup):
         fn()
     ctx.barrier()
@@ -439,9 +451,10 @@ def e2e(ctx, name, steps, warmup):
     wall = (time.perf_counter() - t0) / steps
     ms = ctx.max(ev0.elapsed_time(ev1) / steps)
     ctx.barrier()
-    return {"value": p * ctx.world / (ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": n * p * 4,
-            "d2h_bytes_per_step": n * p * 4, "ms_per_step": ms, "wall_ms_per_step": wall * 1e3,
-            "api": "bulk_prefix_sums_host (pinned host in/out, 2-stream chunked H2D/compute/D2H)",
+    api = "bulk_triangulation_host" if tri else "bulk_prefix_sums_host"
+    return {"value": p * ctx.world / (ms * 1e-3), "unit": UNIT, "h2d_bytes_per_step": in_bytes,
+            "d2h_bytes_per_step": out_bytes, "ms_per_step": ms, "wall_ms_per_step": wall * 1e3,
+            "api": f"{api} (pinned host in/out, 2-stream chunked H2D/compute/D2H)",
             "gpu_launches": bo.launch_count() - c0}
 
 

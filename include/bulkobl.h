@@ -179,9 +179,14 @@ int bulk_transpose(const void *src, void *dst, int64_t rows, int64_t cols, size_
 /* The host->device copy, the computation and the device->host copy are       */
 /* pipelined in chunks of instances over two internal streams; the call       */
 /* returns after the result is in h_dst (it synchronises).  d_buf is a device */
-/* buffer of at least n*p*4 bytes (prefix) / n*n*p*4 + p*4 bytes (OPT) plus   */
-/* the variant's workspace; h_dst may equal h_src (prefix).                   */
+/* buffer of at least bulk_*_host_bytes(...) bytes: the whole input, the      */
+/* (OPT) output vector, and one workspace per internal stream (the two chunk  */
+/* streams never share scratch).  h_dst may equal h_src (prefix).  Errors as  */
+/* for the device entry points; a short d_buf is BO_EINVAL (message names the */
+/* size needed).                                                              */
 /* ------------------------------------------------------------------------- */
+size_t bulk_prefix_sums_host_bytes(int64_t n, int64_t p, int dtype, int layout, int variant);
+size_t bulk_triangulation_host_bytes(int64_t n, int64_t p, int dtype, int layout, int variant);
 int bulk_prefix_sums_host(const void *h_src, void *h_dst, int64_t n, int64_t p, int dtype,
                           int layout, int variant, void *d_buf, size_t d_bytes, void *stream);
 int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, int dtype,

@@ -63,6 +63,8 @@ def lib() -> ctypes.CDLL:
             "bulk_execute": ([vp, i64, vp, sz, vp, i64, i64, i32, i32, i32, vp], i32),
             "bulk_prefix_sums_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_triangulation_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
+            "bulk_prefix_sums_host_bytes": ([i64, i64, i32, i32, i32], sz),
+            "bulk_triangulation_host_bytes": ([i64, i64, i32, i32, i32], sz),
             "bulk_generate_prefix": ([vp, i64, i64, i64, u64, i32, i32, i32, vp], i32),
             "bulk_generate_tri": ([vp, i64, i64, i64, u64, i32, i32, vp], i32),
             "bulk_checksum": ([vp, i64, i64, i64, i32, vp, vp], i32),
@@ -142,6 +144,16 @@ def prefix_sums_variant(n: int, p: int, dtype: int, layout: int, variant: int = 
     return int(lib().bulk_prefix_sums_variant(n, p, dtype, layout, variant, None, None))
 
 
+def prefix_sums_host_bytes(n: int, p: int, dtype: int, layout: int = ROW_WISE, variant: int = AUTO) -> int:
+    """Device buffer size bulk_prefix_sums_host needs (data + per-stream workspace)."""
+    return int(lib().bulk_prefix_sums_host_bytes(n, p, dtype, layout, variant))
+
+
+def triangulation_host_bytes(n: int, p: int, dtype: int, layout: int = ROW_WISE, variant: int = AUTO) -> int:
+    """Device buffer size bulk_triangulation_host needs (weights + output + workspace)."""
+    return int(lib().bulk_triangulation_host_bytes(n, p, dtype, layout, variant))
+
+
 def prefix_sums_host(x_host: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO,
                      out_host: torch.Tensor | None = None, device_buf: torch.Tensor | None = None,
                      stream=None) -> torch.Tensor:
@@ -152,7 +164,7 @@ def prefix_sums_host(x_host: torch.Tensor, layout: int = ROW_WISE, variant: int 
     if out_host is None:
         out_host = torch.empty_like(x_host)
     if device_buf is None:
-        need = n * p * 4 + 2 * prefix_sums_workspace(n, (p + 7) // 8 + 128, dt, layout, variant)
+        need = prefix_sums_host_bytes(n, p, dt, layout, variant)
         device_buf = torch.empty(need, dtype=torch.uint8, device="cuda")
     _check(lib().bulk_prefix_sums_host(x_host.data_ptr(), out_host.data_ptr(), n, p, dt, layout, variant,
                                        device_buf.data_ptr(), device_buf.numel(), _stream(stream)))
@@ -249,8 +261,7 @@ def triangulation_host(c_host: torch.Tensor, layout: int = ROW_WISE, variant: in
     if out_host is None:
         out_host = torch.empty(p, dtype=c_host.dtype).pin_memory()
     if device_buf is None:
-        words = (n - 1) * (n - 2) // 2 if layout in (PACKED_ROW, PACKED_COLUMN) else n * n
-        need = words * p * 4 + p * 4 + triangulation_workspace(n, p, dt, layout, variant)
+        need = triangulation_host_bytes(n, p, dt, layout, variant)
         device_buf = torch.empty(need, dtype=torch.uint8, device="cuda")
     _check(lib().bulk_triangulation_host(c_host.data_ptr(), out_host.data_ptr(), n, p, dt, layout, variant,
                                          device_buf.data_ptr(), device_buf.numel(), _stream(stream)))

@@ -317,6 +317,12 @@ int bulk_checksum(const void *values, int64_t n, int64_t p, int64_t h0, int layo
 }
 
 // ------------------------------------------------------------------ host e2e
+size_t bulk_prefix_sums_host_bytes(int64_t n, int64_t p, int dtype, int layout, int variant) {
+    if (n < 0 || p < 0 || n * p == 0) return 0;
+    const int v = resolve_prefix_variant(n, p, dtype, layout, variant, nullptr, nullptr);
+    return static_cast<size_t>(n) * p * 4 + 2 * prefix_ws(n, host_chunk(p), v);
+}
+
 int bulk_prefix_sums_host(const void *h_src, void *h_dst, int64_t n, int64_t p, int dtype, int layout,
                           int variant, void *d_buf, size_t d_bytes, void *stream) {
     t_err.clear();
@@ -371,6 +377,20 @@ int bulk_prefix_sums_host(const void *h_src, void *h_dst, int64_t n, int64_t p, 
     return cuda_check(cudaStreamSynchronize(caller), "prefix_host: sync");
 }
 
+// Scratch of one chunk stream: the UMM variant keeps a table per instance, so
+// the chunks use disjoint slices of one p-sized workspace; TILED_GLOBAL keeps
+// a table per CTA, so each of the two streams gets its own chunk-sized copy.
+static size_t tri_host_ws(int64_t n, int64_t p, int v) {
+    if (v == BO_TRI_TILED_GLOBAL) return 2 * tri_workspace(n, host_chunk(p), v);
+    return tri_workspace(n, p, v);
+}
+
+size_t bulk_triangulation_host_bytes(int64_t n, int64_t p, int dtype, int layout, int variant) {
+    if (n < 3 || p <= 0 || !valid_tri_layout(layout)) return 0;
+    const int v = resolve_tri_variant(n, p, dtype, layout, variant);
+    return static_cast<size_t>(tri_words(n, layout)) * p * 4 + static_cast<size_t>(p) * 4 + tri_host_ws(n, p, v);
+}
+
 int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, int dtype, int layout,
                             int variant, void *d_buf, size_t d_bytes, void *stream) {
     t_err.clear();
@@ -381,7 +401,7 @@ int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, 
     const int64_t ch = host_chunk(p);
     const size_t nn = static_cast<size_t>(tri_words(n, layout));     // weights per instance
     const size_t c_bytes = nn * p * 4, out_bytes = static_cast<size_t>(p) * 4;
-    const size_t ws_bytes = tri_workspace(n, p, v);
+    const size_t ws_bytes = tri_host_ws(n, p, v);
     if (!d_buf || d_bytes < c_bytes + out_bytes + ws_bytes)
         return fail(BO_EINVAL, "triangulation_host: device buffer too small (need " +
                                    std::to_string(c_bytes + out_bytes + ws_bytes) + " bytes)");
@@ -408,7 +428,9 @@ int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, 
             rc = cuda_check(cudaMemcpy2DAsync(dchunk, pc * 4, hc + p0 * 4, p * 4, pc * 4, nn, cudaMemcpyHostToDevice, s),
                             "tri_host: H2D");
         if (rc) return rc;
-        void *ws = ws_bytes ? dws + static_cast<size_t>(p0) * (n - 1) * (n - 1) * 4 : nullptr;
+        void *ws = nullptr;
+        if (v == BO_TRI_UMM_GLOBAL) ws = dws + static_cast<size_t>(p0) * (n - 1) * (n - 1) * 4;
+        else if (ws_bytes) ws = dws + (k & 1) * (ws_bytes / 2);
         if ((rc = tri_dispatch(dchunk, dout + p0 * 4, n, pc, dtype, layout, v, ws, s))) return rc;
         if ((rc = cuda_check(cudaMemcpyAsync(ho + p0 * 4, dout + p0 * 4, pc * 4, cudaMemcpyDeviceToHost, s),
                              "tri_host: D2H")))

@@ -100,3 +100,20 @@ def test_launch_counter_counts_kernels():
     x = torch.zeros((16, 16), device=DEV)
     bo.prefix_sums(x, bo.ROW_WISE, bo.PS_TRANSPOSED)
     assert bo.launch_count() - before == 3          # transpose, scan, transpose
+
+
+@pytest.mark.parametrize("n,p,variant", [(40, 1500, bo.AUTO), (40, 1500, bo.TRI_TILED_HALF),
+                                         (80, 600, bo.TRI_TILED_GLOBAL), (16, 700, bo.TRI_THREAD_REG)])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+def test_tri_host_entry_point_chunked_variants(n, p, variant, layout):
+    # several chunks in flight on the two internal streams; TILED_GLOBAL gives each stream its own scratch
+    c = bulkgen.tri_input(n, p, seed=n + p, dtype="float32", layout=layout)
+    dt = bo.F32
+    need = bo.triangulation_host_bytes(n, p, dt, layout, variant)
+    assert need >= c.size * 4 + p * 4
+    out = bo.triangulation_host(torch.from_numpy(c).pin_memory(), layout, variant)
+    ref = oracle.bulk_opt(c, layout)
+    assert np.array_equal(out.numpy().view(np.uint32), ref.view(np.uint32))
+    short = torch.empty(need - 4, dtype=torch.uint8, device=DEV)
+    with pytest.raises(bo.BulkError):
+        bo.triangulation_host(torch.from_numpy(c).pin_memory(), layout, variant, device_buf=short)
