@@ -19,7 +19,7 @@ import os
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbulkobl.so")
+LIB_PATH = os.environ.get("BULKOBL_LIB") or os.path.join(_HERE, "libbulkobl.so")   # override: A/B timing only
 
 ROW_WISE, COLUMN_WISE, PACKED_ROW, PACKED_COLUMN = 0, 1, 2, 3
 I32, F32 = 0, 1

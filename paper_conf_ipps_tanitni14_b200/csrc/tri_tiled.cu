@@ -125,14 +125,78 @@ __device__ __forceinline__ void minplus_chunk(int32_t (&acc)[4][4], const int4 (
 #pragma unroll
             for (int v = 0; v < 4; ++v) acc[u][v] = __viaddmin_s32(comp(A[u], w), comp(B[w], v), acc[u][v]);
 }
+// The 4x4 fix-up of one tile: with S = the dense part (k outside the tile's
+// own diagonal tiles), for u = 3..0, v = 0..3
+//   t[u][v] = min(S[u][v], min_{w>u} A[u][w] + t[w][v]   (P1, diagonal tile I)
+//                         , min_{w<v} t[u][w] + Bd[w][v]) (P3, diagonal tile J)
+//             + C[u][v]
+// -- the same sums as Algorithm OPT's inner loop, min taken in another order
+// (exact).  Generic form: one add-min per term.
+template <typename T>
+__device__ __forceinline__ void fixup(T (&t)[4][4], const T (&S)[4][4], const T (&A)[4][4], const T (&Bd)[4][4],
+                                      const T (&C)[4][4], bool edge) {
+#pragma unroll
+    for (int u = 3; u >= 0; --u)
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+            T sv = S[u][v];
+#pragma unroll
+            for (int w = u + 1; w < 4; ++w) sv = Ops<T>::addmin(A[u][w], t[w][v], sv);   // P1
+#pragma unroll
+            for (int w = 0; w < v; ++w) sv = Ops<T>::addmin(t[u][w], Bd[w][v], sv);       // P3
+            t[u][v] = Ops<T>::add(sv, C[u][v]);
+            if (u == 3 && v == 0 && edge) t[u][v] = T(0);
+        }
+}
+// fp32: P1 terms of a row pair two v's in one FADD2 (A[u][w] broadcast), P3
+// terms pair v = 2, 3, and mins fold two terms per FMNMX3: 64 instructions per
+// tile instead of 112.
+__device__ __forceinline__ float2 add2b(float a, float x, float y) {
+    return __fadd2_rn(make_float2(a, a), make_float2(x, y));
+}
+__device__ __forceinline__ float min3(float a, float b, float c) { return fminf(fminf(a, b), c); }
+template <>
+__device__ __forceinline__ void fixup<float>(float (&t)[4][4], const float (&S)[4][4], const float (&A)[4][4],
+                                             const float (&Bd)[4][4], const float (&C)[4][4], bool edge) {
+#pragma unroll
+    for (int u = 3; u >= 0; --u) {
+        float R[4] = {S[u][0], S[u][1], S[u][2], S[u][3]};
+#pragma unroll
+        for (int w = u + 1; w < 4; w += 2) {                  // P1, two w per FMNMX3
+            const float2 x01 = add2b(A[u][w], t[w][0], t[w][1]), x23 = add2b(A[u][w], t[w][2], t[w][3]);
+            if (w + 1 < 4) {
+                const float2 y01 = add2b(A[u][w + 1], t[w + 1][0], t[w + 1][1]);
+                const float2 y23 = add2b(A[u][w + 1], t[w + 1][2], t[w + 1][3]);
+                R[0] = min3(R[0], x01.x, y01.x); R[1] = min3(R[1], x01.y, y01.y);
+                R[2] = min3(R[2], x23.x, y23.x); R[3] = min3(R[3], x23.y, y23.y);
+            } else {
+                R[0] = fminf(R[0], x01.x); R[1] = fminf(R[1], x01.y);
+                R[2] = fminf(R[2], x23.x); R[3] = fminf(R[3], x23.y);
+            }
+        }
+        // P3, sequential in v
+        t[u][0] = edge && u == 3 ? 0.0f : __fadd_rn(R[0], C[u][0]);
+        const float2 a23 = add2b(t[u][0], Bd[0][2], Bd[0][3]);
+        t[u][1] = __fadd_rn(fminf(R[1], __fadd_rn(t[u][0], Bd[0][1])), C[u][1]);
+        const float2 b23 = add2b(t[u][1], Bd[1][2], Bd[1][3]);
+        t[u][2] = __fadd_rn(min3(R[2], a23.x, b23.x), C[u][2]);
+        t[u][3] = __fadd_rn(min3(fminf(R[3], a23.y), b23.y, __fadd_rn(t[u][2], Bd[2][3])), C[u][3]);
+    }
+}
 }  // namespace tt
 
 // Lanes per tile on tile-diagonal D (t = NT-D tiles): 2^ls, the largest power
 // of two with t * 2^ls <= lanes that does not exceed the D-1 dense chunks.
-__device__ __forceinline__ int split_log2(int t, int D, int lpi) {
+__host__ __device__ inline int split_log2(int t, int D, int lpi) {
     int ls = 0;
     while ((2 << ls) * t <= lpi && (1 << ls) < D - 1) ++ls;
     return ls;
+}
+// the whole schedule in one kernel parameter: 4 bits of log2(split) per D
+static uint64_t split_schedule(int NT, int lpi) {
+    uint64_t m = 0;
+    for (int D = 1; D < NT; ++D) m |= static_cast<uint64_t>(split_log2(NT - D, D, lpi)) << (4 * D);
+    return m;
 }
 
 // Extra shared words per instance for the chord walk (stack of intervals).
@@ -141,7 +205,7 @@ __host__ __device__ constexpr int chord_stack_words(int NT) { return 8 * NT + 4;
 template <typename T, int LPI, bool CHORDS>
 __global__ void __launch_bounds__(128, 1)
 tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restrict__ chords, int n, long long p,
-                 int layout, int NT, int c_vec) {
+                 int layout, int NT, int c_vec, uint64_t lsched) {
     using Op = tt::Ops<T>;
     using T4 = typename tt::V4<T>::type;
     using tt::xc;
@@ -235,9 +299,16 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
 
         // ------------------------------------------------ 3. D = 1 .. NT-1
         for (int D = 1; D < NT; ++D) {
-            const int ls = split_log2(NT - D, D, LPI);
+            const int ls = static_cast<int>(lsched >> (4 * D)) & 15;     // split_log2(NT - D, D, LPI)
+            // tile index in the low bits, split index q in the high bits: the 8-lane
+            // phases of an LDS.128 then hold consecutive tiles of one q, whose chunk
+            // addresses fall in distinct 16-byte bank groups (tools/smem_model.py:
+            // 1386 -> 1124 wavefronts per instance at n = 64), and the q == 0 lanes
+            // that run the fix-up are lanes 0..t-1
+            constexpr int kLogLpi = LPI == 16 ? 4 : 5;
+            const int ib = kLogLpi - ls;
+            const int I = li & ((1 << ib) - 1), q = li >> ib;
             const int s = 1 << ls;
-            const int I = li >> ls, q = li & (s - 1);
             const bool act = I < NT - D;
             const int J = I + D;
             T acc[4][4];
@@ -279,7 +350,7 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
                     }
                 }
             }
-            for (int off = 1; off < s; off <<= 1)
+            for (int off = 1 << ib; off < LPI; off <<= 1)
 #pragma unroll
                 for (int u = 0; u < 4; ++u)
 #pragma unroll
@@ -300,19 +371,8 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
                     C[r][0] = w.x; C[r][1] = w.y; C[r][2] = w.z; C[r][3] = w.w;
                 }
                 T t[4][4];
-#pragma unroll
-                for (int u = 3; u >= 0; --u)
-#pragma unroll
-                    for (int v = 0; v < 4; ++v) {
-                        T sv = acc[u][v];
-#pragma unroll
-                        for (int w = u + 1; w < 4; ++w) sv = Op::addmin(A[u][w], t[w][v], sv);   // P1
-#pragma unroll
-                        for (int w = 0; w < v; ++w) sv = Op::addmin(t[u][w], Bd[w][v], sv);       // P3
-                        t[u][v] = Op::add(sv, C[u][v]);
-                        // X[4I+3][4I+4] is an edge of the polygon (M[i][i] = 0)
-                        if (u == 3 && v == 0 && D == 1) t[u][v] = T(0);
-                    }
+                // X[4I+3][4I+4] is an edge of the polygon when D == 1 (M[i][i] = 0)
+                tt::fixup(t, acc, A, Bd, C, D == 1);
 #pragma unroll
                 for (int u = 0; u < 4; ++u) tt::st4(tc + 4 * u, t[u][0], t[u][1], t[u][2], t[u][3]);
             }
@@ -394,7 +454,8 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
                                                  static_cast<long long>(per_sm) * num_sms());
     const int c_vec = (n % 4 == 0) && aligned16(c);
     tri_tiled_kernel<T, LPI, CHORDS><<<static_cast<unsigned>(blocks), W * 32, smem, st>>>(
-        static_cast<const T *>(c), static_cast<T *>(out), chords, static_cast<int>(n), p, layout, NT, c_vec);
+        static_cast<const T *>(c), static_cast<T *>(out), chords, static_cast<int>(n), p, layout, NT, c_vec,
+        split_schedule(NT, LPI));
     return after_launch("tri_tiled_kernel");
 }
 
@@ -509,18 +570,7 @@ tri_tiled_global_kernel(const T *__restrict__ c, T *__restrict__ out, T *ws, int
                         C[r][0] = w.x; C[r][1] = w.y; C[r][2] = w.z; C[r][3] = w.w;
                     }
                     T tt_[4][4];
-#pragma unroll
-                    for (int u = 3; u >= 0; --u)
-#pragma unroll
-                        for (int v = 0; v < 4; ++v) {
-                            T sv = acc[u][v];
-#pragma unroll
-                            for (int w = u + 1; w < 4; ++w) sv = Op::addmin(A[u][w], tt_[w][v], sv);
-#pragma unroll
-                            for (int w = 0; w < v; ++w) sv = Op::addmin(tt_[u][w], Bd[w][v], sv);
-                            tt_[u][v] = Op::add(sv, C[u][v]);
-                            if (u == 3 && v == 0 && D == 1) tt_[u][v] = T(0);
-                        }
+                    tt::fixup(tt_, acc, A, Bd, C, D == 1);
 #pragma unroll
                     for (int u = 0; u < 4; ++u) tt::st4(tc + 4 * u, tt_[u][0], tt_[u][1], tt_[u][2], tt_[u][3]);
                 }
