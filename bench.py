@@ -325,15 +325,28 @@ def measure(ctx, name, steps, warmup, stream, peaks, traffic):
         res["roofline"] = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                            "frac": gbs / peaks["hbm_gbs"]}
     else:
-        ops = addmin_per_instance(wl) * wl["p"]
-        tops = ops / (ms * 1e-3) / 1e12
-        alu_peak = alu_peak_taddmin(peaks, wl["dtype"])
-        gbs = bytes_launch / (ms * 1e-3) / 1e9
-        res["roofline"] = {"bound": "alu", "achieved": tops, "peak": alu_peak, "unit": "T add-min/s",
-                           "frac": tops / alu_peak,
-                           "hbm": {"achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                                   "frac": gbs / peaks["hbm_gbs"]}}
+        res["roofline"] = tri_roofline(wl, ms * steps / max(1, launches), peaks)
     return res, st
+
+
+def tri_roofline(wl, per_launch_ms, peaks):
+    """Triangulation is bounded by whichever roof is slower for its work
+    (SURVEY.md §8 d): HBM for the algorithmic bytes or the ALU for the C(n,3)
+    add-mins.  Returns the binding roof, with the other one alongside."""
+    p = wl["p"]
+    secs = per_launch_ms * 1e-3
+    gbs = algo_bytes_per_instance(wl) * p / secs / 1e9
+    tops = addmin_per_instance(wl) * p / secs / 1e12
+    alu = alu_peak_taddmin(peaks, wl["dtype"])
+    hbm = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": gbs / peaks["hbm_gbs"]}
+    alu_r = {"bound": "alu", "achieved": tops, "peak": alu, "unit": "T add-min/s", "frac": tops / alu}
+    t_hbm = algo_bytes_per_instance(wl) * p / (peaks["hbm_gbs"] * 1e9)
+    t_alu = addmin_per_instance(wl) * p / (alu * 1e12)
+    main, other = (hbm, alu_r) if t_hbm >= t_alu else (alu_r, hbm)
+    out = dict(main)
+    out["other_roof"] = other
+    out["roof_time_us"] = {"hbm": t_hbm * 1e6, "alu": t_alu * 1e6}
+    return out
 
 
 def alu_peak_taddmin(peaks, dtype):
@@ -492,7 +505,7 @@ def run_ours(args, ctx):
     # roofline of the dominant kernel (the only kernel of the step for AUTO)
     per_launch_ms = ms * args.steps / max(1, launches)
     bytes_launch = algo_bytes_per_instance(wl) * wl["p"]
-    if wl["algo"] == "prefix":
+    if wl["algo"] in ("prefix", "exec"):
         ach = bytes_launch / (per_launch_ms * 1e-3) / 1e9
         tr = traffic.get(name, {}).get("dram_bytes_per_launch")
         line["roofline"] = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
@@ -500,11 +513,11 @@ def run_ours(args, ctx):
                             "peak_source": peak_src + " hbm_gbs (burst copy)",
                             "kernel": st["variant"], "algorithmic_bytes_per_launch": bytes_launch}
     else:
-        ops = addmin_per_instance(wl) * wl["p"]
-        ach = ops / (per_launch_ms * 1e-3) / 1e12
-        pk = alu_peak_taddmin(peaks, wl["dtype"])
-        line["roofline"] = {"bound": "alu", "achieved": ach, "peak": pk, "unit": "T add-min/s",
-                            "frac": ach / pk, "traffic": traffic.get(name, {}).get("dram_bytes_per_launch")}
+        line["roofline"] = tri_roofline(wl, per_launch_ms, peaks)
+        line["roofline"]["traffic"] = traffic.get(name, {}).get("dram_bytes_per_launch")
+        line["roofline"]["kernel"] = st["variant"]
+        line["roofline"]["algorithmic_bytes_per_launch"] = algo_bytes_per_instance(wl) * wl["p"]
+        line["roofline"]["addmin_per_launch"] = addmin_per_instance(wl) * wl["p"]
     line["clocks"] = sampler.summary()
     # checksum of each rank's shard, one NCCL all-gather (SURVEY §8 e), off the timed region
     from paper_conf_ipps_tanitni14_b200 import shard

@@ -37,10 +37,17 @@ def up_to_date() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and up_to_date():
-        return LIB
     objdir = os.path.join(HERE, "build")
     os.makedirs(objdir, exist_ok=True)
+    # nvcc also reads NVCC_APPEND_FLAGS (development A/B builds): a change of it forces a rebuild
+    stamp = os.path.join(objdir, "append_flags.txt")
+    extra = os.environ.get("NVCC_APPEND_FLAGS", "")
+    if (open(stamp).read() if os.path.exists(stamp) else "") != extra:
+        force = True
+        with open(stamp, "w") as fh:
+            fh.write(extra)
+    if not force and up_to_date():
+        return LIB
     objs = []
     procs = []
     for src in sources():

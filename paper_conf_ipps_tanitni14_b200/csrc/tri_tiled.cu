@@ -117,6 +117,33 @@ __device__ __forceinline__ void minplus_chunk(float (&acc)[4][4], const float4 (
             }
         }
 }
+// acc = the first chunk's min_w A[u].w + B[w].v (same sums, min order is free)
+__device__ __forceinline__ void minplus_first(float (&acc)[4][4], const float4 (&A)[4], const float4 (&B)[4]) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int v = 0; v < 4; v += 2) {
+            float2 s[4];
+#pragma unroll
+            for (int w = 0; w < 4; ++w) {
+                const float a = comp(A[u], w);
+                s[w] = __fadd2_rn(make_float2(a, a), make_float2(comp(B[w], v), comp(B[w], v + 1)));
+            }
+            acc[u][v] = fminf(fminf(fminf(s[0].x, s[1].x), s[2].x), s[3].x);
+            acc[u][v + 1] = fminf(fminf(fminf(s[0].y, s[1].y), s[2].y), s[3].y);
+        }
+}
+__device__ __forceinline__ void minplus_first(int32_t (&acc)[4][4], const int4 (&A)[4], const int4 (&B)[4]) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int v = 0; v < 4; ++v) {
+            int32_t r = add_wrap(comp(A[u], 0), comp(B[0], v));
+#pragma unroll
+            for (int w = 1; w < 4; ++w) r = __viaddmin_s32(comp(A[u], w), comp(B[w], v), r);
+            acc[u][v] = r;
+        }
+}
 __device__ __forceinline__ void minplus_chunk(int32_t (&acc)[4][4], const int4 (&A)[4], const int4 (&B)[4]) {
 #pragma unroll
     for (int u = 0; u < 4; ++u)
@@ -148,13 +175,15 @@ __device__ __forceinline__ void fixup(T (&t)[4][4], const T (&S)[4][4], const T 
             if (u == 3 && v == 0 && edge) t[u][v] = T(0);
         }
 }
-// fp32: P1 terms of a row pair two v's in one FADD2 (A[u][w] broadcast), P3
-// terms pair v = 2, 3, and mins fold two terms per FMNMX3: 64 instructions per
-// tile instead of 112.
 __device__ __forceinline__ float2 add2b(float a, float x, float y) {
     return __fadd2_rn(make_float2(a, a), make_float2(x, y));
 }
 __device__ __forceinline__ float min3(float a, float b, float c) { return fminf(fminf(a, b), c); }
+// fp32, row-ordered: P1 terms of a row pair two v's in one FADD2 (A[u][w]
+// broadcast), P3 terms pair v = 2, 3, and mins fold two terms per FMNMX3: 64
+// instructions per tile instead of 112.  (A latency-ordered variant -- cells by
+// anti-diagonal, newest terms last, scalar adds -- measured 5% slower: the
+// kernel is bound by issue slots more than by this chain.)
 template <>
 __device__ __forceinline__ void fixup<float>(float (&t)[4][4], const float (&S)[4][4], const float (&A)[4][4],
                                              const float (&Bd)[4][4], const float (&C)[4][4], bool edge) {
@@ -312,43 +341,51 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             const bool act = I < NT - D;
             const int J = I + D;
             T acc[4][4];
-#pragma unroll
-            for (int u = 0; u < 4; ++u)
-#pragma unroll
-                for (int v = 0; v < 4; ++v) acc[u][v] = Op::inf();
-            if (act) {
-                int m = I + 1 + q;
+            int m = I + 1 + q;
+            if (act && m < J) {
                 const T *pa = Z + xc(4 * I, m);                 // A rows 4I+u: pa + 4u
                 const T *pb = Z + xc(4 * m, J);                 // B rows 4m+w: pb + 4w
                 const int db = 16 * s;                          // B: next chunk = 4s rows further down
-                if (m < J) {
-                    // software-pipelined ping-pong: load chunk m+s while computing chunk m
-                    T4 A0[4], B0[4], A1[4], B1[4];
+                // software-pipelined ping-pong: load chunk m+s while computing chunk m;
+                // the first chunk initialises acc (no +inf fill)
+                T4 A0[4], B0[4], A1[4], B1[4];
 #pragma unroll
-                    for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + 4 * u), B0[u] = tt::ld4(pb + 4 * u);
-                    while (true) {
-                        pa += 4 * (4 * m * s + 2 * s * s + 3 * s);   // colbase(m+s) - colbase(m) chunks
-                        pb += db;
-                        m += s;
-                        bool more = m < J;
-                        if (more) {
+                for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + 4 * u), B0[u] = tt::ld4(pb + 4 * u);
+                pa += 4 * (4 * m * s + 2 * s * s + 3 * s);       // colbase(m+s) - colbase(m) chunks
+                pb += db;
+                m += s;
+                bool more = m < J;
+                if (more) {
 #pragma unroll
-                            for (int u = 0; u < 4; ++u) A1[u] = tt::ld4(pa + 4 * u), B1[u] = tt::ld4(pb + 4 * u);
-                        }
-                        tt::minplus_chunk(acc, A0, B0);
-                        if (!more) break;
-                        pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
-                        pb += db;
-                        m += s;
-                        more = m < J;
-                        if (more) {
-#pragma unroll
-                            for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + 4 * u), B0[u] = tt::ld4(pb + 4 * u);
-                        }
-                        tt::minplus_chunk(acc, A1, B1);
-                        if (!more) break;
-                    }
+                    for (int u = 0; u < 4; ++u) A1[u] = tt::ld4(pa + 4 * u), B1[u] = tt::ld4(pb + 4 * u);
                 }
+                tt::minplus_first(acc, A0, B0);
+                while (more) {
+                    pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
+                    pb += db;
+                    m += s;
+                    more = m < J;
+                    if (more) {
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + 4 * u), B0[u] = tt::ld4(pb + 4 * u);
+                    }
+                    tt::minplus_chunk(acc, A1, B1);
+                    if (!more) break;
+                    pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
+                    pb += db;
+                    m += s;
+                    more = m < J;
+                    if (more) {
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) A1[u] = tt::ld4(pa + 4 * u), B1[u] = tt::ld4(pb + 4 * u);
+                    }
+                    tt::minplus_chunk(acc, A0, B0);
+                }
+            } else {
+#pragma unroll
+                for (int u = 0; u < 4; ++u)
+#pragma unroll
+                    for (int v = 0; v < 4; ++v) acc[u][v] = Op::inf();
             }
             for (int off = 1 << ib; off < LPI; off <<= 1)
 #pragma unroll
