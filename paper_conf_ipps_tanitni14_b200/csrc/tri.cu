@@ -85,7 +85,7 @@ tri_thread_reg(const T *__restrict__ c, T *__restrict__ out, long long p) {
 // lane).  Two smem buffers: the next batch's boxes are in flight while the
 // current batch computes.  Only elements up to the last one Algorithm OPT
 // reads are fetched.
-template <typename T, int N, int LAYOUT>
+template <typename T, int N, int LAYOUT, int S>
 __global__ void __launch_bounds__(32)
 tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out, long long p, long long nbatch) {
     using Op = MinPlus<T>;
@@ -95,32 +95,35 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
     constexpr uint32_t kBatchBytes = NB * 4096;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint64_t *bar = reinterpret_cast<uint64_t *>(buf + 2 * kBatchBytes);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(buf + S * kBatchBytes);
     const int t = threadIdx.x;
-    auto issue = [&](long long i) {
+    auto issue = [&](long long i) {                  // batch i of this CTA -> ring slot i % S
         const long long b = blockIdx.x + i * gridDim.x;
-        uint8_t *dst = buf + (i & 1) * kBatchBytes;
-        mbar_arrive_expect_tx(&bar[i & 1], kBatchBytes);
+        if (b >= nbatch) return;
+        const int sl = static_cast<int>(i % S);
+        uint8_t *dst = buf + sl * kBatchBytes;
+        mbar_arrive_expect_tx(&bar[sl], kBatchBytes);
 #pragma unroll
         for (int k = 0; k < NB; ++k) {
-            if (LAYOUT != BO_COLUMN_WISE) tma_load_2d(dst + k * 4096, &cmap, k * 32, static_cast<int>(b * 32), &bar[i & 1]);
-            else tma_load_2d(dst + k * 4096, &cmap, static_cast<int>(b * 32), k * 32, &bar[i & 1]);
+            if (LAYOUT != BO_COLUMN_WISE) tma_load_2d(dst + k * 4096, &cmap, k * 32, static_cast<int>(b * 32), &bar[sl]);
+            else tma_load_2d(dst + k * 4096, &cmap, static_cast<int>(b * 32), k * 32, &bar[sl]);
         }
     };
     if (t == 0) {
         prefetch_tmap(&cmap);
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
+#pragma unroll
+        for (int k = 0; k < S; ++k) mbar_init(&bar[k], 1);
         fence_barrier_init();
-        if (static_cast<long long>(blockIdx.x) < nbatch) issue(0);
+        for (int k = 0; k < (S > 1 ? S - 1 : 1); ++k) issue(k);
     }
     __syncwarp();
     for (long long i = 0;; ++i) {
         const long long b = blockIdx.x + i * gridDim.x;
         if (b >= nbatch) break;
-        if (t == 0 && b + gridDim.x < nbatch) issue(i + 1);   // the other buffer was released last iteration
-        mbar_wait(&bar[i & 1], static_cast<uint32_t>((i >> 1) & 1));
-        const uint8_t *cur = buf + (i & 1) * kBatchBytes;
+        if (S > 1 && t == 0) issue(i + S - 1);              // its slot was released last iteration
+        const int sl = static_cast<int>(i % S);
+        mbar_wait(&bar[sl], static_cast<uint32_t>((i / S) & 1));
+        const uint8_t *cur = buf + sl * kBatchBytes;
         auto cl = [&](int e) -> T {                 // e = dense index a*N + b (compile time)
             if (LAYOUT == BO_PACKED_ROW) {
                 const int a = e / N, b = e % N;
@@ -149,7 +152,8 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
         }
         const long long h = b * 32 + t;
         if (h < p) out[h] = M[1][N - 1];
-        __syncwarp();                                        // buffer i&1 free for batch i+2
+        __syncwarp();                                        // slot i % S free again
+        if (S == 1 && t == 0) issue(i + 1);
     }
 }
 
@@ -338,24 +342,28 @@ size_t tri_workspace(int64_t n, int64_t p, int variant) {
     return 0;
 }
 
+#ifndef BO_REG_TMA_STAGES
+#define BO_REG_TMA_STAGES 2
+#endif
 template <typename T, int N, int LAYOUT>
 static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) {
+    constexpr int S = BO_REG_TMA_STAGES;
     constexpr int NE = (N - 3) * N + N;
     constexpr int NB = (NE + 31) / 32;
-    constexpr size_t smem = 1024 + 2 * NB * 4096 + 16;
+    constexpr size_t smem = 1024 + S * NB * 4096 + 8 * S;
     CUtensorMap map;
     constexpr int K = (N - 1) * (N - 2) / 2;
     const bool ok = LAYOUT == BO_ROW_WISE     ? make_tmap_2d(&map, c, p, N * N, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
                     : LAYOUT == BO_PACKED_ROW ? make_tmap_2d(&map, c, p, K, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
                                               : make_tmap_2d(&map, c, N * N, p, 32, 32, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (!ok) return fail(BO_ECUDA, "triangulation THREAD_REG: cuTensorMapEncodeTiled failed");
-    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_thread_reg_tma<T, N, LAYOUT>), static_cast<int>(smem));
+    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_thread_reg_tma<T, N, LAYOUT, S>), static_cast<int>(smem));
     if (!attr) return fail(BO_ECUDA, "triangulation THREAD_REG: cannot set dynamic smem");
     const long long nbatch = (p + 31) / 32;
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_thread_reg_tma<T, N, LAYOUT>, 32, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_thread_reg_tma<T, N, LAYOUT, S>, 32, smem);
     const long long grid = std::min<long long>(nbatch, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
-    tri_thread_reg_tma<T, N, LAYOUT><<<static_cast<unsigned>(grid), 32, smem, st>>>(map, static_cast<T *>(out), p,
+    tri_thread_reg_tma<T, N, LAYOUT, S><<<static_cast<unsigned>(grid), 32, smem, st>>>(map, static_cast<T *>(out), p,
                                                                                      nbatch);
     return after_launch("tri_thread_reg_tma");
 }

@@ -37,12 +37,15 @@ def t_ms(fn, reps):
 
 def main():
     reps = int(sys.argv[sys.argv.index("--reps") + 1]) if "--reps" in sys.argv else 20
-    cfgs = [(64, 65536, "float32", bo.ROW_WISE, bo.AUTO), (64, 65536, "int32", bo.ROW_WISE, bo.AUTO),
+    small = [(16, 65536, "int32", bo.ROW_WISE, bo.AUTO), (16, 65536, "int32", bo.COLUMN_WISE, bo.AUTO),
+             (16, 65536, "int32", bo.PACKED_ROW, bo.AUTO), (16, 65536, "float32", bo.ROW_WISE, bo.AUTO),
+             (12, 65536, "int32", bo.ROW_WISE, bo.AUTO), (16, 1 << 20, "int32", bo.ROW_WISE, bo.AUTO)]
+    cfgs = small if "--small" in sys.argv else [(64, 65536, "float32", bo.ROW_WISE, bo.AUTO), (64, 65536, "int32", bo.ROW_WISE, bo.AUTO),
             (64, 65536, "float32", bo.COLUMN_WISE, bo.AUTO), (64, 65536, "float32", bo.PACKED_ROW, bo.AUTO),
             (64, 65536, "float32", bo.ROW_WISE, bo.TRI_TILED), (40, 65536, "float32", bo.ROW_WISE, bo.AUTO),
             (33, 65536, "int32", bo.ROW_WISE, bo.AUTO), (64, 65536, "float32", bo.ROW_WISE, "chords")]
-    ids = np.unique(np.linspace(0, 65535, 64).astype(np.int64))
     for n, p, dt, layout, v in cfgs:
+        ids = np.unique(np.linspace(0, p - 1, 64).astype(np.int64))
         c = bo.generate_tri(n, p, 4, getattr(torch, dt), layout)
         if v == "chords":
             fn = lambda: bo.triangulation_chords(c, layout)
