@@ -230,6 +230,15 @@ static uint64_t split_schedule(int NT, int lpi) {
 
 // Extra shared words per instance for the chord walk (stack of intervals).
 __host__ __device__ constexpr int chord_stack_words(int NT) { return 8 * NT + 4; }
+// Shared words between consecutive instance tables.  Two instances per warp
+// (LPI = 16) sit on alternate lanes (slot = lane & 1), so an 8-lane LDS.128
+// phase holds 4 tiles of each; their tables are offset by 16 words (mod 32)
+// so the two halves fall in opposite bank-group halves (tools/smem_model.py,
+// --interleave: 1124 -> 968 wavefronts per instance at n = 64).
+__host__ __device__ constexpr int table_stride(int NT, int ipw) {
+    return ipw == 2 ? 4 * (2 * NT * NT + 3 * NT) + ((16 - 4 * (2 * NT * NT + 3 * NT)) % 32 + 32) % 32
+                    : 4 * (2 * NT * NT + 3 * NT);
+}
 
 template <typename T, int LPI, bool CHORDS>
 __global__ void __launch_bounds__(128, 1)
@@ -241,8 +250,10 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
     constexpr int IPW = 32 / LPI;                       // instances per warp
     extern __shared__ uint8_t smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int slot = lane / LPI, li = lane % LPI;       // instance slot in warp, lane in instance
-    const int words = 4 * tt::colbase(NT);            // per-instance table size
+    // instance slot in the warp and lane within the instance: alternate lanes
+    // for two instances per warp (see table_stride)
+    const int slot = IPW == 2 ? (lane & 1) : 0, li = IPW == 2 ? (lane >> 1) : lane;
+    const int words = table_stride(NT, IPW);             // per-instance table size (+ bank pad)
     const int warps_per_cta = blockDim.x >> 5;
     T *Z = reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warp * IPW + slot) * words;
     int *stk = reinterpret_cast<int *>(reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warps_per_cta) * IPW * words) +
@@ -392,7 +403,7 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
                 for (int u = 0; u < 4; ++u)
 #pragma unroll
                     for (int v = 0; v < 4; ++v)
-                        acc[u][v] = Op::min(acc[u][v], __shfl_xor_sync(0xffffffffu, acc[u][v], off));
+                        acc[u][v] = Op::min(acc[u][v], __shfl_xor_sync(0xffffffffu, acc[u][v], off * IPW));
             if (act && q == 0) {
                 // A[u][w] = X[4I+u][4I+w] (w > u), Bd[w][v] = X[4J+w][4J+v] (v > w),
                 // C[u][v] = c[4I+u][4J+v] (still in the tile's own upper cells)
@@ -439,8 +450,8 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
                 }
 #pragma unroll
                 for (int off = 1; off < LPI; off <<= 1) {
-                    const T ob = __shfl_xor_sync(0xffffffffu, best, off);
-                    const int ok = __shfl_xor_sync(0xffffffffu, kb, off);
+                    const T ob = __shfl_xor_sync(0xffffffffu, best, off * IPW);
+                    const int ok = __shfl_xor_sync(0xffffffffu, kb, off * IPW);
                     if (ob < best || (ob == best && ok < kb)) best = ob, kb = ok;
                 }
                 const int k = kb;
@@ -469,8 +480,8 @@ template <typename T, int LPI, bool CHORDS>
 static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int layout,
                           cudaStream_t st) {
     const int NT = static_cast<int>((n + 3) / 4);
-    const size_t per_inst = static_cast<size_t>(4 * tt::colbase(NT) + (CHORDS ? chord_stack_words(NT) : 0)) * sizeof(T);
     constexpr int IPW = 32 / LPI;
+    const size_t per_inst = static_cast<size_t>(table_stride(NT, IPW) + (CHORDS ? chord_stack_words(NT) : 0)) * sizeof(T);
     // warps per CTA: the W in 1..4 that keeps the most warps resident per SM
     // (shared memory is the limit: 227 KB, 1 KB reserved per CTA)
     int W = 1, best = 0;
