@@ -28,6 +28,11 @@ KEYS = {
     "l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum": "smem_bank_conflicts",
     "smsp__inst_executed_pipe_fma.sum": "pipe_fma_inst",
     "smsp__inst_executed_pipe_alu.sum": "pipe_alu_inst",
+    "sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active": "alu_pct",
+    "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active": "fma_pct",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum": "smem_wavefronts",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed": "smem_pct",
+    "lts__t_sectors.sum": "l2_sectors",
 }
 SCALE = {"Kbyte/block": 1e3, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "byte": 1, "Tbyte": 1e12,
          "nsecond": 1e-9, "usecond": 1e-6, "msecond": 1e-3, "second": 1, "ns": 1e-9, "us": 1e-6, "ms": 1e-3}
@@ -55,6 +60,8 @@ def read(rep):
 def main():
     outdir = sys.argv[1]
     os.makedirs(outdir, exist_ok=True)
+    if len(sys.argv) > 2 and sys.argv[2].startswith("--compare="):
+        return compare(outdir, sys.argv[2].split("=", 1)[1], sys.argv[3:])
     table = ["| capture | kernel | duration (us) | DRAM read (MB) | DRAM write (MB) | DRAM % peak | SM % | "
              "issue active % | warps active % | regs | grid x block | smem/CTA (KB) |",
              "|---|---|---|---|---|---|---|---|---|---|---|---|"]
@@ -75,6 +82,28 @@ def main():
         f.write("\n".join(table) + "\n")
     with open(os.path.join(outdir, "traffic.json"), "w") as f:
         json.dump(traffic, f, indent=1)
+    print("\n".join(table))
+
+
+def compare(outdir, fname, args):
+    """Variant comparison table (pipe/issue/memory utilisation side by side)."""
+    table = ["| capture | kernel | duration (us) | issue active % | ALU pipe % | FMA pipe % | smem wavefronts % | "
+             "DRAM read (MB) | DRAM % peak | L2 bytes (MB) | warps active % | regs |",
+             "|---|---|---|---|---|---|---|---|---|---|---|---|"]
+    for arg in args:
+        name, rep = arg.split("=", 1)
+        if not os.path.exists(rep):
+            table.append(f"| {name} | (no capture) |" + " |" * 10)
+            continue
+        for d in read(rep):
+            k = d["kernel"].split("(")[0].split("<")[0].replace("void ", "").strip()
+            table.append(
+                f"| {name} | `{k}` | {d.get('duration', 0) * 1e6:.1f} | {d.get('issue_active_pct', 0):.1f} | "
+                f"{d.get('alu_pct', 0):.1f} | {d.get('fma_pct', 0):.1f} | {d.get('smem_pct', 0):.1f} | "
+                f"{d.get('dram_read', 0) / 1e6:.1f} | {d.get('dram_pct', 0):.1f} | {d.get('l2_sectors', 0) * 32 / 1e6:.1f} | "
+                f"{d.get('occupancy_pct', 0):.1f} | {d.get('regs', 0):.0f} |")
+    with open(os.path.join(outdir, fname), "w") as f:
+        f.write("\n".join(table) + "\n")
     print("\n".join(table))
 
 
