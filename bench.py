@@ -377,10 +377,10 @@ def cpu_baseline(ctx, name, st, budget_s=12.0):
             return bulkgen.prefix_instances(n, ids, st["seed"], wl["dtype"])
         return bulkgen.tri_instances(n, ids, st["seed"], wl["dtype"])
 
-    def run(x):
+    def run(x, threads=cores):
         if wl["algo"] == "prefix":
-            return oracle.bulk_prefix_sums(x, oracle.ROW_WISE, nthreads=cores)
-        return oracle.bulk_opt(x, oracle.ROW_WISE, nthreads=cores)
+            return oracle.bulk_prefix_sums(x, oracle.ROW_WISE, nthreads=threads)
+        return oracle.bulk_opt(x, oracle.ROW_WISE, nthreads=threads)
 
     # calibrate
     k = 256
@@ -401,6 +401,19 @@ def cpu_baseline(ctx, name, st, budget_s=12.0):
     t0 = time.perf_counter()
     ref = run(x)
     dt = time.perf_counter() - t0
+    reps = 1
+    if dt < 2.0:                             # whole workload in well under 2 s: time repeated passes
+        reps = int(min(512, max(2, 2.0 / max(dt, 1e-6))))
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            run(x)
+        dt = (time.perf_counter() - t0) / reps
+    # one core, like the paper's single-CPU baseline: a ~2 s sample
+    k1 = max(32, min(len(ids), int(2.0 * len(ids) / max(dt * cores, 1e-9))))
+    x1 = x[:k1]
+    t0 = time.perf_counter()
+    run(x1, threads=1)
+    dt1 = time.perf_counter() - t0
     # parity of the sampled instances (GPU output vs oracle)
     loc = torch.from_numpy(ids - st["h0"]).cuda()
     out = st["out"]
@@ -412,8 +425,22 @@ def cpu_baseline(ctx, name, st, budget_s=12.0):
     ok = bool(np.array_equal(g.view(np.uint32), ref.view(np.uint32)))
     return {"value": len(ids) / dt, "unit": UNIT, "cores": cores, "kind": "oracle",
             "sample": f"{len(ids)} of the {p} instances of workload '{name}' (evenly spaced ids), "
-                      f"plain C oracle, {cores} threads, {dt:.1f} s",
+                      f"plain C oracle, {cores} threads, {dt:.3f} s per pass"
+                      + (f" (mean of {reps} passes)" if reps > 1 else ""),
+            "single_core": {"value": k1 / dt1, "unit": UNIT, "cores": 1,
+                            "sample": f"first {k1} instances of the sample, {dt1:.2f} s"},
+            "cpu_model": cpu_model(),
             "gpu_matches_oracle_on_sample": ok}
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 def e2e(ctx, name, steps, warmup):
@@ -577,10 +604,10 @@ def run_reference(args, ctx):
             return bulkgen.prefix_instances(n, ids, wl["seed"], wl["dtype"])
         return bulkgen.tri_instances(n, ids, wl["seed"], wl["dtype"])
 
-    def run(x):
+    def run(x, threads=cores):
         if wl["algo"] == "prefix":
-            return oracle.bulk_prefix_sums(x, oracle.ROW_WISE, nthreads=cores)
-        return oracle.bulk_opt(x, oracle.ROW_WISE, nthreads=cores)
+            return oracle.bulk_prefix_sums(x, oracle.ROW_WISE, nthreads=threads)
+        return oracle.bulk_opt(x, oracle.ROW_WISE, nthreads=threads)
 
     k = 1024
     while True:
