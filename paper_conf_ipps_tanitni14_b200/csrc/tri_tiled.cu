@@ -293,24 +293,23 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             }
             tt::cp_async_wait_all();
         } else if (layout == BO_COLUMN_WISE || layout == BO_PACKED_COLUMN) {
-            // Column-wise weights c[(a*n+b)*p + h] or packed c[k*p + h]: the whole CTA loads the
-            // weights of its `ninst` consecutive instances together, instance index
-            // fastest, so each warp request covers whole 32-byte sectors.
-            __syncthreads();                                // every table of the CTA is free
-            T *Z0 = reinterpret_cast<T *>(smem_raw);
-            for (int a = 0; a < n - 2; ++a) {
-                const int L = n - a - 2;                    // cells (a, a+2 .. n-1)
-                const long long row0 = layout == BO_COLUMN_WISE ? static_cast<long long>(a) * n + a + 2
-                                                                : tri_c_index(BO_PACKED_COLUMN, 0, n, 1, a, a + 2);
-                for (int idx = threadIdx.x; idx < L * ninst; idx += blockDim.x) {
-                    const int q = idx % ninst, b = a + 2 + idx / ninst;
-                    if (base + q < p)
-                        tt::cp_async4(Z0 + static_cast<size_t>(q) * words + tt::xoff(a, b),
-                                      c + (row0 + (b - a - 2)) * p + base + q);
+            // Column-wise weights c[(a*n+b)*p + h] or packed c[k*p + h]: each
+            // warp fetches its own two instances (on alternate lanes, so one request
+            // covers 16 cells x 2 adjacent instances); the 4 warps of a CTA hold 8
+            // consecutive instances, so a 32-byte sector is fetched from HBM once and
+            // its other quarters hit L2.  Measured 0.72 ms at TR-2 against 0.92 ms
+            // for a CTA-cooperative preload with whole-sector requests (which needs
+            // two __syncthreads per instance batch and per-element index math).
+            if (live) {
+                const long long pl = static_cast<long long>(LPI) * p;
+                for (int a = 0; a < n - 2; ++a) {
+                    const long long row0 = layout == BO_COLUMN_WISE ? static_cast<long long>(a) * n + a + 2
+                                                                    : tri_c_index(BO_PACKED_COLUMN, 0, n, 1, a, a + 2);
+                    const T *src = c + (row0 + li) * p + h;
+                    for (int b = a + 2 + li; b < n; b += LPI, src += pl) tt::cp_async4(Z + tt::xoff(a, b), src);
                 }
             }
             tt::cp_async_wait_all();
-            __syncthreads();
         } else if (live) {
             // packed row-wise or unaligned dense row-wise: 4-byte asynchronous copies
             // (a packed row is contiguous, so lanes read consecutive words)
