@@ -155,3 +155,13 @@ def test_max_size_64bit_indexing():
     yc = bo.prefix_sums(xc, bo.COLUMN_WISE)
     got = yc[:, torch.from_numpy(ids).to(DEV)].T.contiguous().cpu().numpy()
     assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("n,p", [(100, 37892), (77, 40000), (64, 38000)])
+def test_column_wise_tma_ring_ragged(dt, n, p):
+    # shapes on the TMA column-wise path (p % 4 == 0, >= 2*128*SMs instances, n >= 64) whose last
+    # 128-instance block and last 32-row chunk are partial: element by element against the oracle
+    x = bulkgen.prefix_input(n, p, seed=n + p, dtype=dt, layout=bulkgen.COLUMN_WISE)
+    got = bo.prefix_sums(torch.from_numpy(x).to(DEV), bo.COLUMN_WISE).cpu().numpy()
+    assert np.array_equal(got.view(np.uint32), oracle.bulk_prefix_sums(x, oracle.COLUMN_WISE).view(np.uint32))
