@@ -5,7 +5,7 @@
 // r <- r + b[i] per instance, so fp32 results are bit-identical to the
 // sequential algorithm.  int32 adds wrap mod 2^32.
 //
-//  ACROSS     column-wise [n][p]: a TMA ring of [32 rows x 128
+//  ACROSS     column-wise [n][p]: a TMA ring of [64 rows x 128
 //             instances] boxes, thread t scans column t in shared memory
 //             (ps_across_tma); or, for short columns / unaligned data, a
 //             thread owns 4 adjacent instances, one 128-bit coalesced
@@ -205,13 +205,30 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
 // scans column t with conflict-free 32-bit shared accesses, in place, and the
 // box is stored back by TMA.  No transposition is involved: this is the
 // paper's column-wise bulk order with HBM streamed by TMA.
+namespace ac {
+#ifndef BO_AC_ROWS
+#define BO_AC_ROWS 64
+#endif
+#ifndef BO_AC_STAGES
+#define BO_AC_STAGES 4
+#endif
+// measured at PS-2 column-wise: 64-row boxes x 4 stages (2 CTAs/SM) 1.349 ms,
+// 32 x 8 1.356, 32 x 4 1.360, 64 x 3 1.356, 16 x 8 1.360
+constexpr int kElems = BO_AC_ROWS;          // rows per box
+constexpr int kStages = BO_AC_STAGES;
+template <int INST> struct Cfg {
+    static constexpr uint32_t kBoxBytes = INST * kElems * 4;
+    static constexpr size_t kSmem = 1024 + kStages * kBoxBytes + kStages * 16;
+};
+}  // namespace ac
+
 template <typename T, int kInst>
 __global__ void __launch_bounds__(kInst)
 ps_across_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant__ CUtensorMap dst_map,
               long long ntiles, int nchunks, int slot) {
-    using fr::kElems;
-    constexpr int kStages = fr::Cfg<kInst>::kStages;
-    constexpr uint32_t kBoxBytes = fr::Cfg<kInst>::kBoxBytes;
+    using ac::kElems;
+    constexpr int kStages = ac::kStages;
+    constexpr uint32_t kBoxBytes = ac::Cfg<kInst>::kBoxBytes;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                                ~uintptr_t(1023));
@@ -395,15 +412,15 @@ int resolve_prefix_variant(int64_t n, int64_t p, int dtype, int layout, int vari
 
 template <typename T, int INST>
 static int launch_across_tma(const T *src, T *dst, int64_t n, int64_t p, cudaStream_t st) {
-    using C = fr::Cfg<INST>;
+    using C = ac::Cfg<INST>;
     CUtensorMap smap, dmap;
-    if (!make_tmap_2d(&smap, src, n, p, fr::kElems, INST, CU_TENSOR_MAP_SWIZZLE_NONE) ||
-        !make_tmap_2d(&dmap, dst, n, p, fr::kElems, INST, CU_TENSOR_MAP_SWIZZLE_NONE))
+    if (!make_tmap_2d(&smap, src, n, p, ac::kElems, INST, CU_TENSOR_MAP_SWIZZLE_NONE) ||
+        !make_tmap_2d(&dmap, dst, n, p, ac::kElems, INST, CU_TENSOR_MAP_SWIZZLE_NONE))
         return fail(BO_ECUDA, "prefix across: cuTensorMapEncodeTiled failed");
     const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&ps_across_tma<T, INST>), static_cast<int>(C::kSmem));
     if (!attr) return fail(BO_ECUDA, "prefix across: cannot set dynamic smem");
     const long long ntiles = (p + INST - 1) / INST;
-    const int nchunks = static_cast<int>((n + fr::kElems - 1) / fr::kElems);
+    const int nchunks = static_cast<int>((n + ac::kElems - 1) / ac::kElems);
     int per_sm = 1;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ps_across_tma<T, INST>, INST, C::kSmem);
     const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
