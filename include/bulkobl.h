@@ -85,10 +85,13 @@ typedef enum {
                                tiles (min-plus blocked product), 5 <= n <= 64     */
     BO_TRI_TILED_HALF = 20, /* as BO_TRI_TILED with 16 lanes per instance (two
                                instances per warp)                                 */
-    BO_TRI_TILED_GLOBAL = 21 /* CTA per instance, same blocked algorithm, table in a
+    BO_TRI_TILED_GLOBAL = 21, /* CTA per instance, same blocked algorithm, table in a
                                per-CTA global workspace slot kept L2-resident
                                (large n, e.g. 512-gons); workspace
                                min(p, #SMs) * 16 * (2T^2 + 3T) bytes, T = ceil(n/4) */
+    BO_TRI_TILED_QUARTER = 22 /* as BO_TRI_TILED with 8 lanes per instance (four
+                               instances per warp; a lane takes several tiles of a
+                               tile-diagonal in turn)                             */
 } bo_variant;
 
 /* ------------------------------------------------------------------------- */

@@ -132,7 +132,7 @@ static int check_tri_args(const void *c, const void *out, int64_t n, int64_t p, 
     if (!valid_tri_layout(layout)) return fail(BO_EINVAL, "triangulation: bad layout");
     if (p > kMaxElems / (n * n)) return fail(BO_EINVAL, "triangulation: n*n*p too large");
     if (p > 0 && (!c || !out)) return fail(BO_EINVAL, "triangulation: NULL pointer");
-    if (variant != BO_AUTO && (variant < BO_TRI_UMM_GLOBAL || variant > BO_TRI_TILED_GLOBAL))
+    if (variant != BO_AUTO && (variant < BO_TRI_UMM_GLOBAL || variant > BO_TRI_TILED_QUARTER))
         return fail(BO_EINVAL, "triangulation: unknown variant");
     return BO_OK;
 }

@@ -332,7 +332,9 @@ int resolve_tri_variant(int64_t n, int64_t p, int dtype, int layout, int variant
     (void)p; (void)dtype; (void)layout;
     if (variant != BO_AUTO) return variant;
     if (n <= 16) return BO_TRI_THREAD_REG;
-    if (tiled_supported(n)) return BO_TRI_TILED_HALF;   // 16 lanes per instance: faster at every n measured
+    // 8 lanes per instance (two tiles per lane on the long tile-diagonals) up to
+    // n = 56 (1.1-1.6x faster than 16 lanes, tools/tri_time.py --cmp); 16 lanes above
+    if (tiled_supported(n)) return n <= 56 ? BO_TRI_TILED_QUARTER : BO_TRI_TILED_HALF;
     return BO_TRI_TILED_GLOBAL;
 }
 
@@ -452,9 +454,10 @@ static int run_tri(const void *c, void *out, int64_t n, int64_t p, int layout, i
             return launch_smem_warp<T>(c, out, n, p, layout, st);
         case BO_TRI_TILED:
         case BO_TRI_TILED_HALF:
+        case BO_TRI_TILED_QUARTER:
             if (!tiled_supported(n)) return fail(BO_EUNSUPPORTED, "triangulation TILED supports 5 <= n <= 64");
             return launch_tri_tiled(c, out, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout,
-                                    variant == BO_TRI_TILED ? 32 : 16, st);
+                                    variant == BO_TRI_TILED ? 32 : variant == BO_TRI_TILED_HALF ? 16 : 8, st);
         case BO_TRI_TILED_GLOBAL:
             return launch_tri_tiled_global(c, out, ws, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout,
                                            st);

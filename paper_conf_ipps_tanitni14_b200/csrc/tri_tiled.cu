@@ -212,6 +212,125 @@ __device__ __forceinline__ void fixup<float>(float (&t)[4][4], const float (&S)[
         t[u][3] = __fadd_rn(min3(fminf(R[3], a23.y), b23.y, __fadd_rn(t[u][2], Bd[2][3])), C[u][3]);
     }
 }
+
+// Dense part of tile (I, J) over chunk-columns m, m + s, ... < J (m < J):
+// software-pipelined ping-pong (load chunk m+s while computing chunk m); the
+// first chunk initialises acc (no +inf fill).
+template <typename T>
+__device__ __forceinline__ void dense_tile(T (&acc)[4][4], const T *Z, int I, int J, int m, int s) {
+    using T4 = typename V4<T>::type;
+    const T *pa = Z + xc(4 * I, m);                 // A rows 4I+u: pa + 4u
+    const T *pb = Z + xc(4 * m, J);                 // B rows 4m+w: pb + 4w
+    const int db = 16 * s;                          // B: next chunk = 4s rows further down
+    T4 A0[4], B0[4], A1[4], B1[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) A0[u] = ld4(pa + 4 * u), B0[u] = ld4(pb + 4 * u);
+    pa += 4 * (4 * m * s + 2 * s * s + 3 * s);       // colbase(m+s) - colbase(m) chunks
+    pb += db;
+    m += s;
+    bool more = m < J;
+    if (more) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) A1[u] = ld4(pa + 4 * u), B1[u] = ld4(pb + 4 * u);
+    }
+    minplus_first(acc, A0, B0);
+    while (more) {
+        pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
+        pb += db;
+        m += s;
+        more = m < J;
+        if (more) {
+#pragma unroll
+            for (int u = 0; u < 4; ++u) A0[u] = ld4(pa + 4 * u), B0[u] = ld4(pb + 4 * u);
+        }
+        minplus_chunk(acc, A1, B1);
+        if (!more) break;
+        pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
+        pb += db;
+        m += s;
+        more = m < J;
+        if (more) {
+#pragma unroll
+            for (int u = 0; u < 4; ++u) A1[u] = ld4(pa + 4 * u), B1[u] = ld4(pb + 4 * u);
+        }
+        minplus_chunk(acc, A0, B0);
+    }
+}
+// Two tiles (I0, I0+D), (I1, I1+D) of one tile-diagonal, all D-1 chunks each
+// (s = 1), interleaved; D == 1 has no dense chunk (acc = +inf).
+template <typename T>
+__device__ __forceinline__ void dense_tile2(T (&acc0)[4][4], T (&acc1)[4][4], const T *Z, int I0, int I1, int D) {
+    using T4 = typename V4<T>::type;
+    if (D < 2) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+#pragma unroll
+            for (int v = 0; v < 4; ++v) acc0[u][v] = acc1[u][v] = Ops<T>::inf();
+        return;
+    }
+    int m0 = I0 + 1, m1 = I1 + 1;
+    const T *pa0 = Z + xc(4 * I0, m0), *pb0 = Z + xc(4 * m0, I0 + D);
+    const T *pa1 = Z + xc(4 * I1, m1), *pb1 = Z + xc(4 * m1, I1 + D);
+    T4 A0[4], B0[4], A1[4], B1[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) A0[u] = ld4(pa0 + 4 * u), B0[u] = ld4(pb0 + 4 * u);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) A1[u] = ld4(pa1 + 4 * u), B1[u] = ld4(pb1 + 4 * u);
+    minplus_first(acc0, A0, B0);
+    minplus_first(acc1, A1, B1);
+    for (int k = 2; k < D; ++k) {
+        pa0 += 4 * (4 * m0 + 5), pa1 += 4 * (4 * m1 + 5);       // colbase(m+1) - colbase(m) = 4m + 5 chunks
+        pb0 += 16, pb1 += 16;
+        ++m0, ++m1;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) A0[u] = ld4(pa0 + 4 * u), B0[u] = ld4(pb0 + 4 * u);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) A1[u] = ld4(pa1 + 4 * u), B1[u] = ld4(pb1 + 4 * u);
+        minplus_chunk(acc0, A0, B0);
+        minplus_chunk(acc1, A1, B1);
+    }
+}
+template <typename T>
+__device__ __forceinline__ void load_fix_operands(const T *Z, int I, int J, T (&A)[4][4], T (&Bd)[4][4], T (&C)[4][4]) {
+    using T4 = typename V4<T>::type;
+    // A[u][w] = X[4I+u][4I+w] (w > u), Bd[w][v] = X[4J+w][4J+v] (v > w),
+    // C[u][v] = c[4I+u][4J+v] (still in the tile's own upper cells)
+    const T *ta = Z + xc(4 * I, I), *tb = Z + xc(4 * J, J), *tc = Z + xc(4 * I, J);
+#pragma unroll
+    for (int r = 0; r < 4; ++r) {
+        const T4 x = ld4(ta + 4 * r), y = ld4(tb + 4 * r), w = ld4(tc + 4 * r);
+        A[r][0] = x.x; A[r][1] = x.y; A[r][2] = x.z; A[r][3] = x.w;
+        Bd[r][0] = y.x; Bd[r][1] = y.y; Bd[r][2] = y.z; Bd[r][3] = y.w;
+        C[r][0] = w.x; C[r][1] = w.y; C[r][2] = w.z; C[r][3] = w.w;
+    }
+}
+// fix-up of tile (I, J = I + D) and store; X[4I+3][4I+4] is an edge of the
+// polygon when D == 1 (M[i][i] = 0)
+template <typename T>
+__device__ __forceinline__ void finish_tile(T *Z, const T (&acc)[4][4], int I, int J, int D) {
+    T A[4][4], Bd[4][4], C[4][4], t[4][4];
+    load_fix_operands(Z, I, J, A, Bd, C);
+    fixup(t, acc, A, Bd, C, D == 1);
+    T *tc = Z + xc(4 * I, J);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) st4(tc + 4 * u, t[u][0], t[u][1], t[u][2], t[u][3]);
+}
+template <typename T>
+__device__ __forceinline__ void finish_tile2(T *Z, const T (&acc0)[4][4], const T (&acc1)[4][4], int I0, int I1, int D,
+                                             bool st1) {
+    T A0[4][4], Bd0[4][4], C0[4][4], t0[4][4], A1[4][4], Bd1[4][4], C1[4][4], t1[4][4];
+    load_fix_operands(Z, I0, I0 + D, A0, Bd0, C0);
+    load_fix_operands(Z, I1, I1 + D, A1, Bd1, C1);
+    fixup(t0, acc0, A0, Bd0, C0, D == 1);
+    fixup(t1, acc1, A1, Bd1, C1, D == 1);
+    T *tc0 = Z + xc(4 * I0, I0 + D), *tc1 = Z + xc(4 * I1, I1 + D);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) st4(tc0 + 4 * u, t0[u][0], t0[u][1], t0[u][2], t0[u][3]);
+    if (st1) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) st4(tc1 + 4 * u, t1[u][0], t1[u][1], t1[u][2], t1[u][3]);
+    }
+}
 }  // namespace tt
 
 // Lanes per tile on tile-diagonal D (t = NT-D tiles): 2^ls, the largest power
@@ -235,9 +354,11 @@ __host__ __device__ constexpr int chord_stack_words(int NT) { return 8 * NT + 4;
 // phase holds 4 tiles of each; their tables are offset by 16 words (mod 32)
 // so the two halves fall in opposite bank-group halves (tools/smem_model.py,
 // --interleave: 1124 -> 968 wavefronts per instance at n = 64).
+// Four instances per warp (LPI = 8) sit on lanes = slot mod 4 with tables
+// 8 words (mod 32) apart, the same idea one level down.
 __host__ __device__ constexpr int table_stride(int NT, int ipw) {
-    return ipw == 2 ? 4 * (2 * NT * NT + 3 * NT) + ((16 - 4 * (2 * NT * NT + 3 * NT)) % 32 + 32) % 32
-                    : 4 * (2 * NT * NT + 3 * NT);
+    return ipw > 1 ? 4 * (2 * NT * NT + 3 * NT) + ((32 / ipw - 4 * (2 * NT * NT + 3 * NT)) % 32 + 32) % 32
+                   : 4 * (2 * NT * NT + 3 * NT);
 }
 
 template <typename T, int LPI, bool CHORDS>
@@ -248,11 +369,13 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
     using T4 = typename tt::V4<T>::type;
     using tt::xc;
     constexpr int IPW = 32 / LPI;                       // instances per warp
+    constexpr int kLogIpw = IPW == 4 ? 2 : IPW == 2 ? 1 : 0;
+    constexpr int kLogLpi = 5 - kLogIpw;
     extern __shared__ uint8_t smem_raw[];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    // instance slot in the warp and lane within the instance: alternate lanes
-    // for two instances per warp (see table_stride)
-    const int slot = IPW == 2 ? (lane & 1) : 0, li = IPW == 2 ? (lane >> 1) : lane;
+    // instance slot in the warp and lane within the instance: the IPW instances
+    // of a warp interleave lane by lane (see table_stride)
+    const int slot = lane & (IPW - 1), li = lane >> kLogIpw;
     const int words = table_stride(NT, IPW);             // per-instance table size (+ bank pad)
     const int warps_per_cta = blockDim.x >> 5;
     T *Z = reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warp * IPW + slot) * words;
@@ -282,13 +405,20 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             // destinations cost one L1 wavefront per lane; TMA boxes would need
             // 128-byte aligned destinations, which the packed table cannot give.
             // LPI = 32: lanes 16..31 take the odd rows.
+            // LPI = 8: each lane takes chunks lm and lm + 8 of every row.
             if (live) {
-                const int lm = li & 15;
-                const T *src = ch + static_cast<long long>(li >> 4) * n;
+                constexpr int RPP = LPI >= 16 ? LPI / 16 : 1;      // rows per pass
+                constexpr int CPL = LPI >= 16 ? 1 : 16 / LPI;      // chunks per lane per row
+                constexpr int LW = LPI >= 16 ? 16 : LPI;           // lanes per row
+                const int lm = li & (LW - 1);
+                const T *src = ch + static_cast<long long>(li / LW) * n;
 #pragma unroll 4
-                for (int a = li >> 4; a < n - 2; a += LPI / 16, src += static_cast<long long>(LPI / 16) * n) {
-                    const int m = ((a + 2) >> 2) + lm;
-                    if (m <= last_chunk) tt::cp_async16(Z + xc(a, m), src + 4 * m, true);
+                for (int a = li / LW; a < n - 2; a += RPP, src += static_cast<long long>(RPP) * n) {
+#pragma unroll
+                    for (int cc = 0; cc < CPL; ++cc) {
+                        const int m = ((a + 2) >> 2) + lm + cc * LW;
+                        if (m <= last_chunk) tt::cp_async16(Z + xc(a, m), src + 4 * m, true);
+                    }
                 }
             }
             tt::cp_async_wait_all();
@@ -320,8 +450,7 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
         __syncwarp();
 
         // ------------------------------------------------ 2. D = 0 (diagonal tiles)
-        if (li < NT) {
-            const int I = li;
+        for (int I = li; I < NT; I += LPI) {
             T *r0 = Z + xc(4 * I, I);                    // rows 4I.. of chunk-column I
             const T4 c0 = tt::ld4(r0), c1 = tt::ld4(r0 + 4);
             const T z = T(0);
@@ -344,53 +473,29 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             // addresses fall in distinct 16-byte bank groups (tools/smem_model.py:
             // 1386 -> 1124 wavefronts per instance at n = 64), and the q == 0 lanes
             // that run the fix-up are lanes 0..t-1
-            constexpr int kLogLpi = LPI == 16 ? 4 : 5;
             const int ib = kLogLpi - ls;
-            const int I = li & ((1 << ib) - 1), q = li >> ib;
+            const int I0 = li & ((1 << ib) - 1), q = li >> ib;
             const int s = 1 << ls;
+            if constexpr (LPI == 8) {
+                // more tiles than lanes (small D, s = 1): lane li takes tiles li and
+                // li + 8 together, interleaved (two independent chains per lane)
+                if (NT - D > LPI) {
+                    const int I1 = I0 + LPI;
+                    const bool act1 = I1 < NT - D;
+                    T acc0[4][4], acc1[4][4];
+                    // a lane without a second tile repeats its first (result discarded)
+                    tt::dense_tile2(acc0, acc1, Z, I0, act1 ? I1 : I0, D);
+                    tt::finish_tile2(Z, acc0, acc1, I0, act1 ? I1 : I0, D, act1);
+                    __syncwarp();
+                    continue;
+                }
+            }
+            const int I = I0;
             const bool act = I < NT - D;
             const int J = I + D;
             T acc[4][4];
-            int m = I + 1 + q;
-            if (act && m < J) {
-                const T *pa = Z + xc(4 * I, m);                 // A rows 4I+u: pa + 4u
-                const T *pb = Z + xc(4 * m, J);                 // B rows 4m+w: pb + 4w
-                const int db = 16 * s;                          // B: next chunk = 4s rows further down
-                // software-pipelined ping-pong: load chunk m+s while computing chunk m;
-                // the first chunk initialises acc (no +inf fill)
-                T4 A0[4], B0[4], A1[4], B1[4];
-#pragma unroll
-                for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + 4 * u), B0[u] = tt::ld4(pb + 4 * u);
-                pa += 4 * (4 * m * s + 2 * s * s + 3 * s);       // colbase(m+s) - colbase(m) chunks
-                pb += db;
-                m += s;
-                bool more = m < J;
-                if (more) {
-#pragma unroll
-                    for (int u = 0; u < 4; ++u) A1[u] = tt::ld4(pa + 4 * u), B1[u] = tt::ld4(pb + 4 * u);
-                }
-                tt::minplus_first(acc, A0, B0);
-                while (more) {
-                    pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
-                    pb += db;
-                    m += s;
-                    more = m < J;
-                    if (more) {
-#pragma unroll
-                        for (int u = 0; u < 4; ++u) A0[u] = tt::ld4(pa + 4 * u), B0[u] = tt::ld4(pb + 4 * u);
-                    }
-                    tt::minplus_chunk(acc, A1, B1);
-                    if (!more) break;
-                    pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
-                    pb += db;
-                    m += s;
-                    more = m < J;
-                    if (more) {
-#pragma unroll
-                        for (int u = 0; u < 4; ++u) A1[u] = tt::ld4(pa + 4 * u), B1[u] = tt::ld4(pb + 4 * u);
-                    }
-                    tt::minplus_chunk(acc, A0, B0);
-                }
+            if (act && I + 1 + q < J) {
+                tt::dense_tile(acc, Z, I, J, I + 1 + q, s);
             } else {
 #pragma unroll
                 for (int u = 0; u < 4; ++u)
@@ -403,26 +508,7 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
 #pragma unroll
                     for (int v = 0; v < 4; ++v)
                         acc[u][v] = Op::min(acc[u][v], __shfl_xor_sync(0xffffffffu, acc[u][v], off * IPW));
-            if (act && q == 0) {
-                // A[u][w] = X[4I+u][4I+w] (w > u), Bd[w][v] = X[4J+w][4J+v] (v > w),
-                // C[u][v] = c[4I+u][4J+v] (still in the tile's own upper cells)
-                T *ta = Z + xc(4 * I, I);
-                T *tb = Z + xc(4 * J, J);
-                T *tc = Z + xc(4 * I, J);
-                T A[4][4], Bd[4][4], C[4][4];
-#pragma unroll
-                for (int r = 0; r < 4; ++r) {
-                    const T4 x = tt::ld4(ta + 4 * r), y = tt::ld4(tb + 4 * r), w = tt::ld4(tc + 4 * r);
-                    A[r][0] = x.x; A[r][1] = x.y; A[r][2] = x.z; A[r][3] = x.w;
-                    Bd[r][0] = y.x; Bd[r][1] = y.y; Bd[r][2] = y.z; Bd[r][3] = y.w;
-                    C[r][0] = w.x; C[r][1] = w.y; C[r][2] = w.z; C[r][3] = w.w;
-                }
-                T t[4][4];
-                // X[4I+3][4I+4] is an edge of the polygon when D == 1 (M[i][i] = 0)
-                tt::fixup(t, acc, A, Bd, C, D == 1);
-#pragma unroll
-                for (int u = 0; u < 4; ++u) tt::st4(tc + 4 * u, t[u][0], t[u][1], t[u][2], t[u][3]);
-            }
+            if (act && q == 0) tt::finish_tile(Z, acc, I, J, D);
             __syncwarp();
         }
         if (live && li == 0) out[h] = Z[tt::xoff(0, n - 1)];   // X[0][n-1] = Algorithm OPT's M[1,n-1]
@@ -506,14 +592,16 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
     return after_launch("tri_tiled_kernel");
 }
 
-// lpi: lanes per instance (BO_TRI_TILED = 32, BO_TRI_TILED_HALF = 16)
+// lpi: lanes per instance (BO_TRI_TILED = 32, BO_TRI_TILED_HALF = 16, BO_TRI_TILED_QUARTER = 8)
 int launch_tri_tiled(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int lpi,
                      cudaStream_t st) {
     if (dtype == BO_F32)
         return lpi == 16 ? launch_tiled_t<float, 16, false>(c, out, nullptr, n, p, layout, st)
-                         : launch_tiled_t<float, 32, false>(c, out, nullptr, n, p, layout, st);
+               : lpi == 8 ? launch_tiled_t<float, 8, false>(c, out, nullptr, n, p, layout, st)
+                          : launch_tiled_t<float, 32, false>(c, out, nullptr, n, p, layout, st);
     return lpi == 16 ? launch_tiled_t<int32_t, 16, false>(c, out, nullptr, n, p, layout, st)
-                     : launch_tiled_t<int32_t, 32, false>(c, out, nullptr, n, p, layout, st);
+           : lpi == 8 ? launch_tiled_t<int32_t, 8, false>(c, out, nullptr, n, p, layout, st)
+                      : launch_tiled_t<int32_t, 32, false>(c, out, nullptr, n, p, layout, st);
 }
 
 // NEXT-1: values and the chords of an optimal triangulation (16 lanes per instance)

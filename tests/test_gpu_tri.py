@@ -22,14 +22,14 @@ def _variants(n):
     if n <= 18:
         v.append(bo.TRI_THREAD_REG)
     if 5 <= n <= 64:
-        v += [bo.TRI_TILED, bo.TRI_TILED_HALF]
+        v += [bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_TILED_QUARTER]
     return v
 
 
 def _supported(n, variant):
-    if variant in (bo.TRI_TILED, bo.TRI_TILED_HALF) and n > 64:
+    if variant in (bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_TILED_QUARTER) and n > 64:
         return False
-    if variant in (bo.TRI_TILED, bo.TRI_TILED_HALF):
+    if variant in (bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_TILED_QUARTER):
         try:
             bo.triangulation(torch.zeros((1, n, n), device=DEV), bo.ROW_WISE, bo.TRI_TILED)
         except bo.BulkError as e:
@@ -103,8 +103,8 @@ def test_tr2_full_config(layout):
     assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32))
 
 
-@pytest.mark.parametrize("variant", [bo.TRI_SMEM_WARP, bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_TILED_GLOBAL,
-                                     bo.TRI_UMM_GLOBAL])
+@pytest.mark.parametrize("variant", [bo.TRI_SMEM_WARP, bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_TILED_QUARTER,
+                                     bo.TRI_TILED_GLOBAL, bo.TRI_UMM_GLOBAL])
 def test_tr2_variants_agree_full_size(variant):
     n, p = 64, 65536
     c = bo.generate_tri(n, p, 4, torch.float32, bo.ROW_WISE)

@@ -97,6 +97,7 @@ def test_workspace_and_variant_queries(L):
     assert bo.prefix_sums_variant(32, 2 ** 22, bo.I32, bo.ROW_WISE) == bo.PS_FUSED_ROW
     assert bo.triangulation_variant(16, 100, bo.I32, bo.ROW_WISE) == bo.TRI_THREAD_REG
     assert bo.triangulation_variant(64, 100, bo.F32, bo.ROW_WISE) == bo.TRI_TILED_HALF
+    assert bo.triangulation_variant(40, 100, bo.F32, bo.ROW_WISE) == bo.TRI_TILED_QUARTER
     assert bo.triangulation_variant(100, 100, bo.F32, bo.ROW_WISE) == bo.TRI_TILED_GLOBAL
 
 

@@ -40,7 +40,10 @@ def main():
     small = [(16, 65536, "int32", bo.ROW_WISE, bo.AUTO), (16, 65536, "int32", bo.COLUMN_WISE, bo.AUTO),
              (16, 65536, "int32", bo.PACKED_ROW, bo.AUTO), (16, 65536, "float32", bo.ROW_WISE, bo.AUTO),
              (12, 65536, "int32", bo.ROW_WISE, bo.AUTO), (16, 1 << 20, "int32", bo.ROW_WISE, bo.AUTO)]
-    cfgs = small if "--small" in sys.argv else [(64, 65536, "float32", bo.ROW_WISE, bo.AUTO), (64, 65536, "int32", bo.ROW_WISE, bo.AUTO),
+    if "--cmp" in sys.argv:     # --cmp n,dtype,layout,v1/v2/...  (variant numbers)
+        n_, dt_, lay_, vs_ = sys.argv[sys.argv.index("--cmp") + 1].split(",")
+        small = [(int(n_), 65536, dt_, int(lay_), int(v)) for v in vs_.split("/")]
+    cfgs = small if ("--small" in sys.argv or "--cmp" in sys.argv) else [(64, 65536, "float32", bo.ROW_WISE, bo.AUTO), (64, 65536, "int32", bo.ROW_WISE, bo.AUTO),
             (64, 65536, "float32", bo.COLUMN_WISE, bo.AUTO), (64, 65536, "float32", bo.PACKED_ROW, bo.AUTO),
             (64, 65536, "float32", bo.ROW_WISE, bo.TRI_TILED), (40, 65536, "float32", bo.ROW_WISE, bo.AUTO),
             (33, 65536, "int32", bo.ROW_WISE, bo.AUTO), (64, 65536, "float32", bo.ROW_WISE, "chords")]
