@@ -388,7 +388,6 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
 
     const long long inst_stride = static_cast<long long>(gridDim.x) * warps_per_cta * IPW;
     const long long nn = static_cast<long long>(n) * n;
-    const int last_chunk = (n - 1) >> 2;
 
     const int ninst = warps_per_cta * IPW;              // consecutive instances per CTA pass
     for (long long base = static_cast<long long>(blockIdx.x) * ninst; base < p; base += inst_stride) {
@@ -398,26 +397,44 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
         // Only the weights Algorithm OPT reads (b >= a+2) are fetched.
         if (layout == BO_ROW_WISE && c_vec) {
             const T *ch = c + (live ? h : 0) * nn;
-            // Row a: lane li copies 16-byte chunk m0(a) + li of row a (only chunks
-            // holding b >= a+2), so one warp request reads whole contiguous rows.
-            // Asynchronous (cp.async): measured faster than 128-bit loads + stores
-            // (0.46 vs 0.56 ms at TR-2) even though the scattered shared-memory
-            // destinations cost one L1 wavefront per lane; TMA boxes would need
-            // 128-byte aligned destinations, which the packed table cannot give.
-            // LPI = 32: lanes 16..31 take the odd rows.
-            // LPI = 8: each lane takes chunks lm and lm + 8 of every row.
-            if (live) {
-                constexpr int RPP = LPI >= 16 ? LPI / 16 : 1;      // rows per pass
-                constexpr int CPL = LPI >= 16 ? 1 : 16 / LPI;      // chunks per lane per row
-                constexpr int LW = LPI >= 16 ? 16 : LPI;           // lanes per row
-                const int lm = li & (LW - 1);
-                const T *src = ch + static_cast<long long>(li / LW) * n;
+            // Chunk-column m of the table holds rows a <= 4m+1 (those with some
+            // b >= a+2 in columns 4m..4m+3): R(m) = min(4m+2, n-2) consecutive 16-byte
+            // cells in shared memory, one 16-byte piece per row (stride n) in global.
+            // Lanes own column pairs (m, NT-1-m) -- equal row counts -- and stride the
+            // rows by RS, so the loop is pointer increments and one asynchronous copy
+            // (cp.async; measured faster than 128-bit loads + stores, 0.46 vs 0.56 ms
+            // at TR-2; TMA boxes would need 128-byte aligned destinations, which the
+            // packed table cannot give).
+            // LPI = 8 keeps whole-row requests (lane li takes chunks li, li+8 of a
+            // row): with four instances per warp the scattered column-pair requests
+            // measured slower (n = 40: 0.13 -> 0.18 ms).
+            if (LPI == 8 && live) {
+                constexpr int LW = LPI < 16 ? LPI : 16;
+                const int last_chunk = (n - 1) >> 2;
+                const T *src = ch;
 #pragma unroll 4
-                for (int a = li / LW; a < n - 2; a += RPP, src += static_cast<long long>(RPP) * n) {
+                for (int a = 0; a < n - 2; ++a, src += n) {
 #pragma unroll
-                    for (int cc = 0; cc < CPL; ++cc) {
-                        const int m = ((a + 2) >> 2) + lm + cc * LW;
+                    for (int cc = 0; cc < 16 / LW; ++cc) {
+                        const int m = ((a + 2) >> 2) + li + cc * LW;
                         if (m <= last_chunk) tt::cp_async16(Z + xc(a, m), src + 4 * m, true);
+                    }
+                }
+            } else if (live) {
+                const int np = (NT + 1) >> 1;                        // column pairs
+                const int RS = LPI >= 4 * np ? 4 : LPI >= 2 * np ? 2 : 1;
+                if (li < np * RS) {
+                    const int pp = li % np, r = li / np;
+#pragma unroll 1
+                    for (int side = 0; side < 2; ++side) {
+                        const int m = side ? NT - 1 - pp : pp;
+                        if (side && m == pp) break;
+                        const int rows = min(4 * m + 2, n - 2);
+                        T *dst = Z + xc(r, m);
+                        const T *src = ch + static_cast<long long>(r) * n + 4 * m;
+#pragma unroll 4
+                        for (int a = r; a < rows; a += RS, dst += 4 * RS, src += static_cast<long long>(RS) * n)
+                            tt::cp_async16(dst, src, true);
                     }
                 }
             }
