@@ -37,6 +37,20 @@
 
 namespace bo {
 
+#ifdef BO_TRI_CLOCK
+// development instrumentation: cycles per phase (slot 0 = preload, 1 = D=0,
+// 1+D = tile-diagonal D), summed over the instances of lane 0 of every warp
+__device__ unsigned long long g_tri_clock[72];
+#define BO_CLK_MARK(slot)                                                             \
+    do {                                                                              \
+        const long long t_ = clock64();                                               \
+        if (lane == 0) atomicAdd(&g_tri_clock[(slot)], static_cast<unsigned long long>(t_ - clk_)); \
+        clk_ = clock64();                                                             \
+    } while (0)
+#else
+#define BO_CLK_MARK(slot) do {} while (0)
+#endif
+
 namespace tt {
 template <typename T>
 struct Ops;
@@ -290,16 +304,29 @@ __device__ __forceinline__ void dense_tile2(T (&acc0)[4][4], T (&acc1)[4][4], co
         minplus_chunk(acc1, A1, B1);
     }
 }
+// The upper part of a diagonal tile (I, I) after step D = 0:
+// X[4I][4I+1..3] = (0, t02, t03), X[4I+1][4I+2..3] = (0, t13), X[4I+2][4I+3] = 0.
+// The lane that fixes up row block I (lane I) computed it itself and keeps it
+// in registers (d[0..2] = t02, t03, t13) instead of reloading it every step.
 template <typename T>
-__device__ __forceinline__ void load_fix_operands(const T *Z, int I, int J, T (&A)[4][4], T (&Bd)[4][4], T (&C)[4][4]) {
+__device__ __forceinline__ void diag_upper(T (&A)[4][4], const T (&d)[3]) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int v = 0; v < 4; ++v) A[u][v] = T(0);
+    A[0][2] = d[0]; A[0][3] = d[1]; A[1][3] = d[2];
+}
+template <typename T>
+__device__ __forceinline__ void load_fix_operands(const T *Z, int I, int J, const T (&d)[3], T (&A)[4][4],
+                                                  T (&Bd)[4][4], T (&C)[4][4]) {
     using T4 = typename V4<T>::type;
-    // A[u][w] = X[4I+u][4I+w] (w > u), Bd[w][v] = X[4J+w][4J+v] (v > w),
+    // A[u][w] = X[4I+u][4I+w] (w > u; registers), Bd[w][v] = X[4J+w][4J+v] (v > w),
     // C[u][v] = c[4I+u][4J+v] (still in the tile's own upper cells)
-    const T *ta = Z + xc(4 * I, I), *tb = Z + xc(4 * J, J), *tc = Z + xc(4 * I, J);
+    diag_upper(A, d);
+    const T *tb = Z + xc(4 * J, J), *tc = Z + xc(4 * I, J);
 #pragma unroll
     for (int r = 0; r < 4; ++r) {
-        const T4 x = ld4(ta + 4 * r), y = ld4(tb + 4 * r), w = ld4(tc + 4 * r);
-        A[r][0] = x.x; A[r][1] = x.y; A[r][2] = x.z; A[r][3] = x.w;
+        const T4 y = ld4(tb + 4 * r), w = ld4(tc + 4 * r);
         Bd[r][0] = y.x; Bd[r][1] = y.y; Bd[r][2] = y.z; Bd[r][3] = y.w;
         C[r][0] = w.x; C[r][1] = w.y; C[r][2] = w.z; C[r][3] = w.w;
     }
@@ -307,9 +334,9 @@ __device__ __forceinline__ void load_fix_operands(const T *Z, int I, int J, T (&
 // fix-up of tile (I, J = I + D) and store; X[4I+3][4I+4] is an edge of the
 // polygon when D == 1 (M[i][i] = 0)
 template <typename T>
-__device__ __forceinline__ void finish_tile(T *Z, const T (&acc)[4][4], int I, int J, int D) {
+__device__ __forceinline__ void finish_tile(T *Z, const T (&acc)[4][4], int I, int J, int D, const T (&d)[3]) {
     T A[4][4], Bd[4][4], C[4][4], t[4][4];
-    load_fix_operands(Z, I, J, A, Bd, C);
+    load_fix_operands(Z, I, J, d, A, Bd, C);
     fixup(t, acc, A, Bd, C, D == 1);
     T *tc = Z + xc(4 * I, J);
 #pragma unroll
@@ -317,10 +344,10 @@ __device__ __forceinline__ void finish_tile(T *Z, const T (&acc)[4][4], int I, i
 }
 template <typename T>
 __device__ __forceinline__ void finish_tile2(T *Z, const T (&acc0)[4][4], const T (&acc1)[4][4], int I0, int I1, int D,
-                                             bool st1) {
+                                             bool st1, const T (&d0)[3], const T (&d1)[3]) {
     T A0[4][4], Bd0[4][4], C0[4][4], t0[4][4], A1[4][4], Bd1[4][4], C1[4][4], t1[4][4];
-    load_fix_operands(Z, I0, I0 + D, A0, Bd0, C0);
-    load_fix_operands(Z, I1, I1 + D, A1, Bd1, C1);
+    load_fix_operands(Z, I0, I0 + D, d0, A0, Bd0, C0);
+    load_fix_operands(Z, I1, I1 + D, st1 ? d1 : d0, A1, Bd1, C1);
     fixup(t0, acc0, A0, Bd0, C0, D == 1);
     fixup(t1, acc1, A1, Bd1, C1, D == 1);
     T *tc0 = Z + xc(4 * I0, I0 + D), *tc1 = Z + xc(4 * I1, I1 + D);
@@ -393,6 +420,9 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
     for (long long base = static_cast<long long>(blockIdx.x) * ninst; base < p; base += inst_stride) {
         const long long h = base + warp * IPW + slot;
         const bool live = h < p;
+#ifdef BO_TRI_CLOCK
+        long long clk_ = clock64();
+#endif
         // ------------------------------------------------ 1. c -> upper table
         // Only the weights Algorithm OPT reads (b >= a+2) are fetched.
         if (layout == BO_ROW_WISE && c_vec) {
@@ -465,9 +495,14 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             tt::cp_async_wait_all();
         }
         __syncwarp();
+        BO_CLK_MARK(0);
 
         // ------------------------------------------------ 2. D = 0 (diagonal tiles)
-        for (int I = li; I < NT; I += LPI) {
+        T dg0[3] = {T(0), T(0), T(0)}, dg1[3] = {T(0), T(0), T(0)};   // diag tiles li, li + LPI (upper part)
+#pragma unroll
+        for (int k = 0; k < (LPI < 16 ? 2 : 1); ++k) {
+            const int I = li + k * LPI;
+            if (I >= NT) break;
             T *r0 = Z + xc(4 * I, I);                    // rows 4I.. of chunk-column I
             const T4 c0 = tt::ld4(r0), c1 = tt::ld4(r0 + 4);
             const T z = T(0);
@@ -479,8 +514,11 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             tt::st4(r0 + 4, z, z, z, t13);
             tt::st4(r0 + 8, z, z, z, z);
             tt::st4(r0 + 12, z, z, z, z);
+            T(&dg)[3] = k == 0 ? dg0 : dg1;
+            dg[0] = t02; dg[1] = t03; dg[2] = t13;
         }
         __syncwarp();
+        BO_CLK_MARK(1);
 
         // ------------------------------------------------ 3. D = 1 .. NT-1
         for (int D = 1; D < NT; ++D) {
@@ -502,8 +540,9 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
                     T acc0[4][4], acc1[4][4];
                     // a lane without a second tile repeats its first (result discarded)
                     tt::dense_tile2(acc0, acc1, Z, I0, act1 ? I1 : I0, D);
-                    tt::finish_tile2(Z, acc0, acc1, I0, act1 ? I1 : I0, D, act1);
+                    tt::finish_tile2(Z, acc0, acc1, I0, act1 ? I1 : I0, D, act1, dg0, dg1);
                     __syncwarp();
+                    BO_CLK_MARK(1 + D);
                     continue;
                 }
             }
@@ -525,10 +564,12 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
 #pragma unroll
                     for (int v = 0; v < 4; ++v)
                         acc[u][v] = Op::min(acc[u][v], __shfl_xor_sync(0xffffffffu, acc[u][v], off * IPW));
-            if (act && q == 0) tt::finish_tile(Z, acc, I, J, D);
+            if (act && q == 0) tt::finish_tile(Z, acc, I, J, D, dg0);   // q == 0: I == li
             __syncwarp();
+            BO_CLK_MARK(1 + D);
         }
         if (live && li == 0) out[h] = Z[tt::xoff(0, n - 1)];   // X[0][n-1] = Algorithm OPT's M[1,n-1]
+
         if constexpr (CHORDS) {
             // NEXT-1: read the optimal triangulation off the finished table.
             // Visit sub-polygons (a, b) depth first, left part first; the split of
@@ -577,6 +618,18 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
 }
 
 int tiled_supported(int64_t n) { return n >= 3 && n <= 64; }
+
+#ifdef BO_TRI_CLOCK
+}  // namespace bo
+extern "C" int bulk_debug_tri_clock(unsigned long long *host72, int reset) {
+    if (reset) {
+        unsigned long long z[72] = {};
+        return cudaMemcpyToSymbol(bo::g_tri_clock, z, sizeof z) == cudaSuccess ? 0 : -3;
+    }
+    return cudaMemcpyFromSymbol(host72, bo::g_tri_clock, 72 * sizeof(unsigned long long)) == cudaSuccess ? 0 : -3;
+}
+namespace bo {
+#endif
 
 template <typename T, int LPI, bool CHORDS>
 static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int layout,
