@@ -18,3 +18,6 @@ prof ps2_across ps_across prefix 1024 1048576 float32 1 1
 prof transpose transpose_tma transpose 1024 1048576 int32 0 0
 prof tr2_tiled tri_tiled tri 64 65536 float32 0 20
 prof tr1_reg tri_thread_reg tri 16 65536 int32 0 18
+prof tr2_tiled8 tri_tiled tri 64 65536 float32 0 22
+prof tr40_tiled8 tri_tiled tri 40 65536 float32 0 22
+prof tr40_tiled16 tri_tiled tri 40 65536 float32 0 20
