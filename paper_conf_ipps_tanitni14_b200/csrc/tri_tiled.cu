@@ -40,7 +40,7 @@ namespace bo {
 #ifdef BO_TRI_CLOCK
 // development instrumentation: cycles per phase (slot 0 = preload, 1 = D=0,
 // 1+D = tile-diagonal D), summed over the instances of lane 0 of every warp
-__device__ unsigned long long g_tri_clock[72];
+__device__ unsigned long long g_tri_clock[160];   // 80 + 4D + k: sub-phases of step D
 #define BO_CLK_MARK(slot)                                                             \
     do {                                                                              \
         const long long t_ = clock64();                                               \
@@ -390,6 +390,84 @@ __host__ __device__ constexpr int table_stride(int NT, int ipw) {
                    : 4 * (2 * NT * NT + 3 * NT);
 }
 
+// Step 1 of an instance: c -> upper table.  Only the weights Algorithm OPT
+// reads (b >= a+2) are fetched; waits for its own copies.
+template <typename T, int LPI, bool WAIT = true>
+__device__ __forceinline__ void preload_table(T *Z, const T *__restrict__ c, long long h, bool live, int n,
+                                              long long p, int layout, int NT, int c_vec, int li) {
+    using tt::xc;
+    const long long nn = static_cast<long long>(n) * n;
+    if (layout == BO_ROW_WISE && c_vec) {
+        const T *ch = c + (live ? h : 0) * nn;
+        // Chunk-column m of the table holds rows a <= 4m+1 (those with some
+        // b >= a+2 in columns 4m..4m+3): R(m) = min(4m+2, n-2) consecutive 16-byte
+        // cells in shared memory, one 16-byte piece per row (stride n) in global.
+        // Lanes own column pairs (m, NT-1-m) -- equal row counts -- and stride the
+        // rows by RS, so the loop is pointer increments and one asynchronous copy
+        // (cp.async; measured faster than 128-bit loads + stores, 0.46 vs 0.56 ms
+        // at TR-2; TMA boxes would need 128-byte aligned destinations, which the
+        // packed table cannot give).
+        // LPI = 8 keeps whole-row requests (lane li takes chunks li, li+8 of a
+        // row): with four instances per warp the scattered column-pair requests
+        // measured slower (n = 40: 0.13 -> 0.18 ms).
+        if (LPI == 8 && live) {
+            constexpr int LW = LPI < 16 ? LPI : 16;
+            const int last_chunk = (n - 1) >> 2;
+            const T *src = ch;
+#pragma unroll 4
+            for (int a = 0; a < n - 2; ++a, src += n) {
+#pragma unroll
+                for (int cc = 0; cc < 16 / LW; ++cc) {
+                    const int m = ((a + 2) >> 2) + li + cc * LW;
+                    if (m <= last_chunk) tt::cp_async16(Z + xc(a, m), src + 4 * m, true);
+                }
+            }
+        } else if (live) {
+            const int np = (NT + 1) >> 1;                        // column pairs
+            const int RS = LPI >= 4 * np ? 4 : LPI >= 2 * np ? 2 : 1;
+            if (li < np * RS) {
+                const int pp = li % np, r = li / np;
+#pragma unroll 1
+                for (int side = 0; side < 2; ++side) {
+                    const int m = side ? NT - 1 - pp : pp;
+                    if (side && m == pp) break;
+                    const int rows = min(4 * m + 2, n - 2);
+                    T *dst = Z + xc(r, m);
+                    const T *src = ch + static_cast<long long>(r) * n + 4 * m;
+#pragma unroll 4
+                    for (int a = r; a < rows; a += RS, dst += 4 * RS, src += static_cast<long long>(RS) * n)
+                        tt::cp_async16(dst, src, true);
+                }
+            }
+        }
+        if (WAIT) tt::cp_async_wait_all();
+    } else if (layout == BO_COLUMN_WISE || layout == BO_PACKED_COLUMN) {
+        // Column-wise weights c[(a*n+b)*p + h] or packed c[k*p + h]: each
+        // warp fetches its own two instances (on alternate lanes, so one request
+        // covers 16 cells x 2 adjacent instances); the 4 warps of a CTA hold 8
+        // consecutive instances, so a 32-byte sector is fetched from HBM once and
+        // its other quarters hit L2.  Measured 0.72 ms at TR-2 against 0.92 ms
+        // for a CTA-cooperative preload with whole-sector requests (which needs
+        // two __syncthreads per instance batch and per-element index math).
+        if (live) {
+            const long long pl = static_cast<long long>(LPI) * p;
+            for (int a = 0; a < n - 2; ++a) {
+                const long long row0 = layout == BO_COLUMN_WISE ? static_cast<long long>(a) * n + a + 2
+                                                                : tri_c_index(BO_PACKED_COLUMN, 0, n, 1, a, a + 2);
+                const T *src = c + (row0 + li) * p + h;
+                for (int b = a + 2 + li; b < n; b += LPI, src += pl) tt::cp_async4(Z + tt::xoff(a, b), src);
+            }
+        }
+        if (WAIT) tt::cp_async_wait_all();
+    } else if (live) {
+        // packed row-wise or unaligned dense row-wise: 4-byte asynchronous copies
+        // (a packed row is contiguous, so lanes read consecutive words)
+        for (int a = 0; a < n - 2; ++a)
+            for (int b = a + 2 + li; b < n; b += LPI) tt::cp_async4(Z + tt::xoff(a, b), c + tri_c_index(layout, h, n, p, a, b));
+        if (WAIT) tt::cp_async_wait_all();
+    }
+}
+
 template <typename T, int LPI, bool CHORDS>
 __global__ void __launch_bounds__(128, 1)
 tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restrict__ chords, int n, long long p,
@@ -426,76 +504,7 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
         long long clk_ = clock64();
 #endif
         // ------------------------------------------------ 1. c -> upper table
-        // Only the weights Algorithm OPT reads (b >= a+2) are fetched.
-        if (layout == BO_ROW_WISE && c_vec) {
-            const T *ch = c + (live ? h : 0) * nn;
-            // Chunk-column m of the table holds rows a <= 4m+1 (those with some
-            // b >= a+2 in columns 4m..4m+3): R(m) = min(4m+2, n-2) consecutive 16-byte
-            // cells in shared memory, one 16-byte piece per row (stride n) in global.
-            // Lanes own column pairs (m, NT-1-m) -- equal row counts -- and stride the
-            // rows by RS, so the loop is pointer increments and one asynchronous copy
-            // (cp.async; measured faster than 128-bit loads + stores, 0.46 vs 0.56 ms
-            // at TR-2; TMA boxes would need 128-byte aligned destinations, which the
-            // packed table cannot give).
-            // LPI = 8 keeps whole-row requests (lane li takes chunks li, li+8 of a
-            // row): with four instances per warp the scattered column-pair requests
-            // measured slower (n = 40: 0.13 -> 0.18 ms).
-            if (LPI == 8 && live) {
-                constexpr int LW = LPI < 16 ? LPI : 16;
-                const int last_chunk = (n - 1) >> 2;
-                const T *src = ch;
-#pragma unroll 4
-                for (int a = 0; a < n - 2; ++a, src += n) {
-#pragma unroll
-                    for (int cc = 0; cc < 16 / LW; ++cc) {
-                        const int m = ((a + 2) >> 2) + li + cc * LW;
-                        if (m <= last_chunk) tt::cp_async16(Z + xc(a, m), src + 4 * m, true);
-                    }
-                }
-            } else if (live) {
-                const int np = (NT + 1) >> 1;                        // column pairs
-                const int RS = LPI >= 4 * np ? 4 : LPI >= 2 * np ? 2 : 1;
-                if (li < np * RS) {
-                    const int pp = li % np, r = li / np;
-#pragma unroll 1
-                    for (int side = 0; side < 2; ++side) {
-                        const int m = side ? NT - 1 - pp : pp;
-                        if (side && m == pp) break;
-                        const int rows = min(4 * m + 2, n - 2);
-                        T *dst = Z + xc(r, m);
-                        const T *src = ch + static_cast<long long>(r) * n + 4 * m;
-#pragma unroll 4
-                        for (int a = r; a < rows; a += RS, dst += 4 * RS, src += static_cast<long long>(RS) * n)
-                            tt::cp_async16(dst, src, true);
-                    }
-                }
-            }
-            tt::cp_async_wait_all();
-        } else if (layout == BO_COLUMN_WISE || layout == BO_PACKED_COLUMN) {
-            // Column-wise weights c[(a*n+b)*p + h] or packed c[k*p + h]: each
-            // warp fetches its own two instances (on alternate lanes, so one request
-            // covers 16 cells x 2 adjacent instances); the 4 warps of a CTA hold 8
-            // consecutive instances, so a 32-byte sector is fetched from HBM once and
-            // its other quarters hit L2.  Measured 0.72 ms at TR-2 against 0.92 ms
-            // for a CTA-cooperative preload with whole-sector requests (which needs
-            // two __syncthreads per instance batch and per-element index math).
-            if (live) {
-                const long long pl = static_cast<long long>(LPI) * p;
-                for (int a = 0; a < n - 2; ++a) {
-                    const long long row0 = layout == BO_COLUMN_WISE ? static_cast<long long>(a) * n + a + 2
-                                                                    : tri_c_index(BO_PACKED_COLUMN, 0, n, 1, a, a + 2);
-                    const T *src = c + (row0 + li) * p + h;
-                    for (int b = a + 2 + li; b < n; b += LPI, src += pl) tt::cp_async4(Z + tt::xoff(a, b), src);
-                }
-            }
-            tt::cp_async_wait_all();
-        } else if (live) {
-            // packed row-wise or unaligned dense row-wise: 4-byte asynchronous copies
-            // (a packed row is contiguous, so lanes read consecutive words)
-            for (int a = 0; a < n - 2; ++a)
-                for (int b = a + 2 + li; b < n; b += LPI) tt::cp_async4(Z + tt::xoff(a, b), c + tri_c_index(layout, h, n, p, a, b));
-            tt::cp_async_wait_all();
-        }
+        preload_table<T, LPI>(Z, c, h, live, n, p, layout, NT, c_vec, li);
         __syncwarp();
         BO_CLK_MARK(0);
 
@@ -560,15 +569,18 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
 #pragma unroll
                     for (int v = 0; v < 4; ++v) acc[u][v] = Op::inf();
             }
+            BO_CLK_MARK(80 + 4 * D);
             for (int off = 1 << ib; off < LPI; off <<= 1)
 #pragma unroll
                 for (int u = 0; u < 4; ++u)
 #pragma unroll
                     for (int v = 0; v < 4; ++v)
                         acc[u][v] = Op::min(acc[u][v], __shfl_xor_sync(0xffffffffu, acc[u][v], off * IPW));
+            BO_CLK_MARK(81 + 4 * D);
             if (act && q == 0) tt::finish_tile(Z, acc, I, J, D, dg0);   // q == 0: I == li
+            BO_CLK_MARK(82 + 4 * D);
             __syncwarp();
-            BO_CLK_MARK(1 + D);
+            BO_CLK_MARK(83 + 4 * D);
         }
         if (live && li == 0) out[h] = Z[tt::xoff(0, n - 1)];   // X[0][n-1] = Algorithm OPT's M[1,n-1]
 
@@ -623,12 +635,12 @@ int tiled_supported(int64_t n) { return n >= 3 && n <= 64; }
 
 #ifdef BO_TRI_CLOCK
 }  // namespace bo
-extern "C" int bulk_debug_tri_clock(unsigned long long *host72, int reset) {
+extern "C" int bulk_debug_tri_clock(unsigned long long *host160, int reset) {
     if (reset) {
-        unsigned long long z[72] = {};
+        unsigned long long z[160] = {};
         return cudaMemcpyToSymbol(bo::g_tri_clock, z, sizeof z) == cudaSuccess ? 0 : -3;
     }
-    return cudaMemcpyFromSymbol(host72, bo::g_tri_clock, 72 * sizeof(unsigned long long)) == cudaSuccess ? 0 : -3;
+    return cudaMemcpyFromSymbol(host160, bo::g_tri_clock, 160 * sizeof(unsigned long long)) == cudaSuccess ? 0 : -3;
 }
 namespace bo {
 #endif
