@@ -376,8 +376,6 @@ static uint64_t split_schedule(int NT, int lpi) {
     return m;
 }
 
-// Extra shared words per instance for the chord walk (stack of intervals).
-__host__ __device__ constexpr int chord_stack_words(int NT) { return 8 * NT + 4; }
 // Shared words between consecutive instance tables.  Two instances per warp
 // (LPI = 16) sit on alternate lanes (slot = lane & 1), so an 8-lane LDS.128
 // phase holds 4 tiles of each; their tables are offset by 16 words (mod 32)
@@ -486,8 +484,6 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
     const int words = table_stride(NT, IPW);             // per-instance table size (+ bank pad)
     const int warps_per_cta = blockDim.x >> 5;
     T *Z = reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warp * IPW + slot) * words;
-    int *stk = reinterpret_cast<int *>(reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warps_per_cta) * IPW * words) +
-               static_cast<size_t>(warp * IPW + slot) * chord_stack_words(NT);
 
     // zero the table once: padding cells then stay finite forever
     for (int i = li; i < words; i += LPI) Z[i] = T(0);
@@ -592,39 +588,53 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             // with the same fp32 adds.  Each split emits (a, k) then (k, b) when
             // that part has >= 3 vertices.  Every instance has n-2 splits, so all
             // lanes of the warp run the same number of iterations.
-            int sp = 2, t = 0;
-            if (li == 0) stk[0] = 0, stk[1] = n - 1;
-            __syncwarp();
+            // The walk state is uniform over the instance's lanes (the argmin is
+            // all-reduced) and lives in registers: the pending right parts (k, b)
+            // are disjoint and ordered (k_last < b_last <= ... < b_first), so the
+            // stack is two 64-bit masks of their starts and ends, and a pop takes
+            // the lowest set bit of each.
+            int a = 0, b = n - 1, t = 0;
+            unsigned long long pend_k = 0, pend_b = 0;
             int16_t *oc = chords + (live ? h : 0) * 2LL * (n - 3);
+            // candidate j of lane li is k = a+1+li+LPI*j: the min is xor-all-reduced,
+            // then the smallest k attaining it is the lowest lane of the first j whose
+            // ballot (this instance's lanes only) is non-empty
+            constexpr int KJ = (64 + LPI - 1) / LPI;
+            const unsigned own = IPW == 1 ? 0xffffffffu : (IPW == 2 ? 0x55555555u : 0x11111111u) << slot;
             for (int it = 0; it < n - 2; ++it) {
-                sp -= 2;
-                const int a = stk[sp], b = stk[sp + 1];
+                T r[KJ];
                 T best = Op::inf();
-                int kb = n;
-                for (int k = a + 1 + li; k < b; k += LPI) {
-                    const T r = Op::add(Z[tt::xoff(a, k)], Z[tt::xoff(k, b)]);
-                    if (r < best) best = r, kb = k;
+#pragma unroll
+                for (int j = 0; j < KJ; ++j) {
+                    const int k = a + 1 + li + LPI * j;
+                    r[j] = k < b ? Op::add(Z[tt::xoff(a, k)], Z[tt::xoff(k, b)]) : Op::inf();
+                    best = Op::min(best, r[j]);
                 }
 #pragma unroll
-                for (int off = 1; off < LPI; off <<= 1) {
-                    const T ob = __shfl_xor_sync(0xffffffffu, best, off * IPW);
-                    const int ok = __shfl_xor_sync(0xffffffffu, kb, off * IPW);
-                    if (ob < best || (ob == best && ok < kb)) best = ob, kb = ok;
+                for (int off = 1; off < LPI; off <<= 1) best = Op::min(best, __shfl_xor_sync(0xffffffffu, best, off * IPW));
+                int k = n;
+#pragma unroll
+                for (int j = KJ - 1; j >= 0; --j) {
+                    const unsigned bal = __ballot_sync(0xffffffffu, a + 1 + li + LPI * j < b && r[j] == best) & own;
+                    if (bal) k = a + 1 + ((__ffs(bal) - 1) >> (IPW == 4 ? 2 : IPW == 2 ? 1 : 0)) + LPI * j;
                 }
-                const int k = kb;
                 const bool left = k - a >= 2, right = b - k >= 2;
-                __syncwarp();
-                if (li == 0) {
-                    if (right) stk[sp] = k, stk[sp + 1] = b;
-                    if (left) stk[sp + 2 * right] = a, stk[sp + 2 * right + 1] = k;
-                    if (live) {
-                        if (left) oc[2 * t] = static_cast<int16_t>(a), oc[2 * t + 1] = static_cast<int16_t>(k);
-                        if (right) oc[2 * (t + left)] = static_cast<int16_t>(k), oc[2 * (t + left) + 1] = static_cast<int16_t>(b);
-                    }
+                if (li == 0 && live) {
+                    if (left) *reinterpret_cast<uint32_t *>(oc + 2 * t) = static_cast<uint32_t>(a) | (static_cast<uint32_t>(k) << 16);
+                    if (right) *reinterpret_cast<uint32_t *>(oc + 2 * (t + left)) = static_cast<uint32_t>(k) | (static_cast<uint32_t>(b) << 16);
                 }
-                sp += 2 * (left + right);
                 t += left + right;
-                __syncwarp();
+                if (left) {
+                    if (right) pend_k |= 1ull << k, pend_b |= 1ull << b;   // (k, b) after the left part
+                    b = k;
+                } else if (right) {
+                    a = k;
+                } else if (pend_k) {                        // leaf: resume at the innermost pending part
+                    a = __ffsll(static_cast<long long>(pend_k)) - 1;
+                    b = __ffsll(static_cast<long long>(pend_b)) - 1;
+                    pend_k &= pend_k - 1;
+                    pend_b &= pend_b - 1;
+                }
             }
         }
         __syncwarp();
@@ -650,7 +660,7 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
                           cudaStream_t st) {
     const int NT = static_cast<int>((n + 3) / 4);
     constexpr int IPW = 32 / LPI;
-    const size_t per_inst = static_cast<size_t>(table_stride(NT, IPW) + (CHORDS ? chord_stack_words(NT) : 0)) * sizeof(T);
+    const size_t per_inst = static_cast<size_t>(table_stride(NT, IPW)) * sizeof(T);
     // warps per CTA: the W in 1..4 that keeps the most warps resident per SM
     // (shared memory is the limit: 227 KB, 1 KB reserved per CTA)
     int W = 1, best = 0;
