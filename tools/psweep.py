@@ -1,12 +1,11 @@
 #!/usr/bin/env python
 """configs[4]: p-sweep 2^10..2^22 for both algorithms on one GPU (AUTO variants,
-device-resident inputs, CUDA events, 3 warm-ups, median of 10, L2 flushed when
-the input is smaller than 2x L2).  Each point also checks a handful of sampled
+device-resident inputs, timed like bench.py: inputs smaller than 2x L2 rotate
+over copies that together exceed it, 20 steps back to back between two events).  Each point also checks a handful of sampled
 instances against the oracle (this is a dev tool; it may use oracle/).
 Prints one JSON line per point.   python tools/psweep.py [--max-log2 22]"""
 import json
 import os
-import statistics
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -18,23 +17,28 @@ import bulkgen  # noqa: E402
 import oracle  # noqa: E402
 import paper_conf_ipps_tanitni14_b200 as bo  # noqa: E402
 
-FLUSH = torch.empty(256 * 2 ** 20 // 4, dtype=torch.int32, device="cuda")
+L2 = 126 * 2 ** 20
 
 
-def med_ms(fn, flush, reps=10):
-    for _ in range(3):
-        fn()
-    ts = []
-    for _ in range(reps):
-        if flush:
-            FLUSH.fill_(1)
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record()
-        fn()
-        b.record()
-        torch.cuda.synchronize()
-        ts.append(a.elapsed_time(b))
-    return statistics.median(ts)
+def rot_ms(step, in_bytes, steps=20):
+    """Per-step ms the way bench.py times it: the step rotates over enough
+    input copies to exceed 2x L2 (step(i) uses copy i mod copies) and K steps
+    run back to back between two events."""
+    for i in range(3):
+        step(i)
+    torch.cuda.synchronize()
+    torch.cuda._sleep(int(0.01 * 2e9))
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for i in range(steps):
+        step(i)
+    b.record()
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / steps
+
+
+def copies(in_bytes):
+    return 1 if in_bytes >= 2 * L2 else -(-2 * L2 // in_bytes) + 1
 
 
 def main():
@@ -49,22 +53,24 @@ def main():
             if algo == "prefix":
                 x = bo.generate_prefix(n, p, 5, tdt, bo.ROW_WISE)
                 y = torch.empty_like(x)
-                ms = med_ms(lambda: bo.prefix_sums(x, bo.ROW_WISE, out=y), n * p * 4 < 2 ** 28)
+                xs = [x] + [x.clone() for _ in range(copies(n * p * 4) - 1)]
+                ms = rot_ms(lambda i: bo.prefix_sums(xs[i % len(xs)], bo.ROW_WISE, out=y), n * p * 4)
                 got = y[torch.from_numpy(ids).cuda()].cpu().numpy()
                 ref = oracle.bulk_prefix_sums(bulkgen.prefix_instances(n, ids, 5, dt), oracle.ROW_WISE)
                 bytes_ = 2 * n * p * 4
                 variant = bo.VARIANT_NAMES[bo.prefix_sums_variant(n, p, bo.I32 if dt == "int32" else bo.F32, 0)]
                 extra = {"GBps": bytes_ / ms / 1e6}
-                del x, y
+                del x, y, xs
             else:
                 c = bo.generate_tri(n, p, 5, tdt, bo.ROW_WISE)
                 out = torch.empty(p, dtype=tdt, device="cuda")
-                ms = med_ms(lambda: bo.triangulation(c, bo.ROW_WISE, out=out), n * n * p * 4 < 2 ** 28)
+                cs = [c] + [c.clone() for _ in range(copies(n * n * p * 4) - 1)]
+                ms = rot_ms(lambda i: bo.triangulation(cs[i % len(cs)], bo.ROW_WISE, out=out), n * n * p * 4)
                 got = out[torch.from_numpy(ids).cuda()].cpu().numpy()
                 ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 5, dt), oracle.ROW_WISE)
                 variant = bo.VARIANT_NAMES[bo.triangulation_variant(n, p, bo.I32 if dt == "int32" else bo.F32, 0)]
                 extra = {"T_addmin_s": n * (n - 1) * (n - 2) // 6 * p / ms / 1e9}
-                del c, out
+                del c, out, cs
             ok = bool(np.array_equal(np.ascontiguousarray(got).view(np.uint32), ref.view(np.uint32)))
             torch.cuda.empty_cache()
             print(json.dumps(dict(algo=algo, n=n, dtype=dt, p=p, variant=variant, ms=ms, inst_per_s=p / ms * 1e3,
