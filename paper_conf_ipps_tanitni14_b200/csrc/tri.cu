@@ -77,26 +77,33 @@ tri_thread_reg(const T *__restrict__ c, T *__restrict__ out, long long p) {
     out[h] = M[1][N - 1];
 }
 
-// THREAD_REG fed by TMA: persistent one-warp CTAs; a batch = 32 instances,
-// whose weights are staged in shared memory by cp.async.bulk.tensor boxes of
-// [32 instances x 32 elements] (row-wise c: box = 32 consecutive elements of
-// 32 instances, 128B-swizzled, read back as conflict-free 128-bit chunks;
-// column-wise c: box = 32 elements x 32 consecutive instances, one word per
-// lane).  Two smem buffers: the next batch's boxes are in flight while the
-// current batch computes.  Only elements up to the last one Algorithm OPT
+// THREAD_REG fed by TMA: persistent CTAs of W warps sharing a ring of S batch
+// slots; a batch = 32 instances (one per lane), whose weights are staged in
+// shared memory by cp.async.bulk.tensor boxes of [32 instances x 32 elements]
+// (row-wise c: box = 32 consecutive elements of 32 instances, 128B-swizzled,
+// read back as conflict-free 128-bit chunks; column-wise c: box = 32 elements
+// x 32 consecutive instances, one word per lane).  Batch i of the CTA goes to
+// slot i % S and is computed by warp i % W; when a warp finishes batch i it
+// issues batch i + S into the slot it just released, so S - W batches are in
+// flight while W compute.  (Measured: p = 2^20 156 us with W = 2, S = 4 against
+// 161 us with one-warp CTAs; p = 65536 is DRAM-bound either way, 14.4 us.)  Only elements up to the last one Algorithm OPT
 // reads are fetched.
-template <typename T, int N, int LAYOUT, int S>
-__global__ void __launch_bounds__(32)
+template <typename T, int N, int LAYOUT, int S, int W>
+__global__ void __launch_bounds__(32 * W)
 tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out, long long p, long long nbatch) {
     using Op = MinPlus<T>;
     constexpr int NE = LAYOUT == BO_PACKED_ROW ? (N - 1) * (N - 2) / 2   // packed: every weight is read
                                                : (N - 3) * N + N;        // c[N-3][N-1] is the last one read
     constexpr int NB = (NE + 31) / 32;
     constexpr uint32_t kBatchBytes = NB * 4096;
+    // slot i % S of batch i is then always one of warp i % W's own slots: a warp
+    // can never wait on (or refill) a slot whose previous batch another warp
+    // still holds, so one full barrier per slot and its phase parity suffice
+    static_assert(S % W == 0 && S / W >= 1, "each warp owns S / W ring slots");
     extern __shared__ uint8_t smem_raw[];
     uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     uint64_t *bar = reinterpret_cast<uint64_t *>(buf + S * kBatchBytes);
-    const int t = threadIdx.x;
+    const int t = threadIdx.x & 31, warp = threadIdx.x >> 5;
     auto issue = [&](long long i) {                  // batch i of this CTA -> ring slot i % S
         const long long b = blockIdx.x + i * gridDim.x;
         if (b >= nbatch) return;
@@ -109,18 +116,18 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
             else tma_load_2d(dst + k * 4096, &cmap, static_cast<int>(b * 32), k * 32, &bar[sl]);
         }
     };
-    if (t == 0) {
+    if (threadIdx.x == 0) {
         prefetch_tmap(&cmap);
 #pragma unroll
         for (int k = 0; k < S; ++k) mbar_init(&bar[k], 1);
         fence_barrier_init();
-        for (int k = 0; k < (S > 1 ? S - 1 : 1); ++k) issue(k);
+        for (int k = 0; k < S; ++k) issue(k);
     }
-    __syncwarp();
-    for (long long i = 0;; ++i) {
+    if (W > 1) __syncthreads();
+    else __syncwarp();
+    for (long long i = warp;; i += W) {
         const long long b = blockIdx.x + i * gridDim.x;
         if (b >= nbatch) break;
-        if (S > 1 && t == 0) issue(i + S - 1);              // its slot was released last iteration
         const int sl = static_cast<int>(i % S);
         mbar_wait(&bar[sl], static_cast<uint32_t>((i / S) & 1));
         const uint8_t *cur = buf + sl * kBatchBytes;
@@ -152,11 +159,10 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
         }
         const long long h = b * 32 + t;
         if (h < p) out[h] = M[1][N - 1];
-        __syncwarp();                                        // slot i % S free again
-        if (S == 1 && t == 0) issue(i + 1);
+        __syncwarp();                                        // every lane is done with slot i % S
+        if (t == 0) issue(i + S);
     }
 }
-
 
 // THREAD_REG on packed row-wise weights (NEXT-4): a batch of 32 consecutive
 // instances is one contiguous run of 32*K words, moved by a single 1-D bulk
@@ -344,12 +350,17 @@ size_t tri_workspace(int64_t n, int64_t p, int variant) {
     return 0;
 }
 
+// ring geometry of the TMA-fed THREAD_REG kernel: W warps per CTA (one CTA per
+// SM), S batch slots of NB*4 KB
 #ifndef BO_REG_TMA_STAGES
-#define BO_REG_TMA_STAGES 2
+#define BO_REG_TMA_STAGES 4
+#endif
+#ifndef BO_REG_TMA_WARPS
+#define BO_REG_TMA_WARPS 2
 #endif
 template <typename T, int N, int LAYOUT>
 static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) {
-    constexpr int S = BO_REG_TMA_STAGES;
+    constexpr int S = BO_REG_TMA_STAGES, W = BO_REG_TMA_WARPS;
     constexpr int NE = (N - 3) * N + N;
     constexpr int NB = (NE + 31) / 32;
     constexpr size_t smem = 1024 + S * NB * 4096 + 8 * S;
@@ -359,14 +370,15 @@ static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) 
                     : LAYOUT == BO_PACKED_ROW ? make_tmap_2d(&map, c, p, K, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
                                               : make_tmap_2d(&map, c, N * N, p, 32, 32, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (!ok) return fail(BO_ECUDA, "triangulation THREAD_REG: cuTensorMapEncodeTiled failed");
-    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_thread_reg_tma<T, N, LAYOUT, S>), static_cast<int>(smem));
+    auto kern = tri_thread_reg_tma<T, N, LAYOUT, S, W>;
+    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(kern), static_cast<int>(smem));
     if (!attr) return fail(BO_ECUDA, "triangulation THREAD_REG: cannot set dynamic smem");
     const long long nbatch = (p + 31) / 32;
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_thread_reg_tma<T, N, LAYOUT, S>, 32, smem);
-    const long long grid = std::min<long long>(nbatch, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
-    tri_thread_reg_tma<T, N, LAYOUT, S><<<static_cast<unsigned>(grid), 32, smem, st>>>(map, static_cast<T *>(out), p,
-                                                                                     nbatch);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * W, smem);
+    // enough CTAs that every warp of every resident CTA has a batch
+    const long long grid = std::min<long long>((nbatch + W - 1) / W, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
+    kern<<<static_cast<unsigned>(grid), 32 * W, smem, st>>>(map, static_cast<T *>(out), p, nbatch);
     return after_launch("tri_thread_reg_tma");
 }
 
