@@ -10,6 +10,7 @@
 
 #include <atomic>
 #include <string>
+#include <utility>
 
 #include "../../include/bulkobl.h"
 
@@ -22,10 +23,39 @@ int cuda_check(cudaError_t e, const char *what);
 extern std::atomic<uint64_t> g_launches;
 inline void count_launch(uint64_t k = 1) { g_launches.fetch_add(k, std::memory_order_relaxed); }
 
-// After a <<<>>> launch: record it and turn a launch error into BO_ECUDA.
+// After a launch: record it and turn a launch error into BO_ECUDA.
 inline int after_launch(const char *what) {
     count_launch();
     return cuda_check(cudaGetLastError(), what);
+}
+
+// Programmatic dependent launch (PDL).  Every kernel is launched with
+// cudaLaunchAttributeProgrammaticStreamSerialization and begins with
+// pdl_begin(): it lets the next kernel in the stream launch as soon as all of
+// its own CTAs have started (griddepcontrol.launch_dependents) and waits for
+// the previous kernel to complete and its memory to be visible
+// (griddepcontrol.wait) before it touches global memory.  Stream order is
+// kept -- nothing is read or written before the predecessor has finished --
+// but launch latency and the predecessor's tail overlap (measured on B200,
+// tools/micro/pdl_gap.cu: a 128 KB kernel 3.5 -> 1.2 us per launch back to
+// back, a 16 MB one 8.2 -> 5.7 us).  Without the attribute both are no-ops.
+__device__ __forceinline__ void pdl_begin() {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+}
+template <typename... KArgs, typename... Args>
+inline void launch(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args &&...args) {
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);   // errors: after_launch()
 }
 
 // Opt a kernel into `bytes` of dynamic shared memory on the current device;

@@ -25,6 +25,7 @@ __device__ __forceinline__ float ex_sub(float a, float b) { return __fsub_rn(a, 
 template <typename T, int LAYOUT>
 __global__ void __launch_bounds__(ex::kThreads)
 exec_kernel(const int4 *__restrict__ prog, long long t, T *mem, long long msize, long long p) {
+    pdl_begin();
     extern __shared__ uint8_t smem_raw[];
     T *R = reinterpret_cast<T *>(smem_raw) + threadIdx.x;     // r[x] at R[x * kThreads]
     const long long j = blockIdx.x * static_cast<long long>(ex::kThreads) + threadIdx.x;
@@ -65,11 +66,11 @@ int launch_exec(const void *prog, int64_t t, void *mem, int64_t msize, int64_t p
     const unsigned grid = static_cast<unsigned>((p + ex::kThreads - 1) / ex::kThreads);
     const int4 *pg = static_cast<const int4 *>(prog);
     if (dtype == BO_F32) {
-        if (layout == BO_ROW_WISE) exec_kernel<float, BO_ROW_WISE><<<grid, ex::kThreads, smem, st>>>(pg, t, static_cast<float *>(mem), msize, p);
-        else exec_kernel<float, BO_COLUMN_WISE><<<grid, ex::kThreads, smem, st>>>(pg, t, static_cast<float *>(mem), msize, p);
+        if (layout == BO_ROW_WISE) launch(exec_kernel<float, BO_ROW_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<float *>(mem), msize, p);
+        else launch(exec_kernel<float, BO_COLUMN_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<float *>(mem), msize, p);
     } else {
-        if (layout == BO_ROW_WISE) exec_kernel<int32_t, BO_ROW_WISE><<<grid, ex::kThreads, smem, st>>>(pg, t, static_cast<int32_t *>(mem), msize, p);
-        else exec_kernel<int32_t, BO_COLUMN_WISE><<<grid, ex::kThreads, smem, st>>>(pg, t, static_cast<int32_t *>(mem), msize, p);
+        if (layout == BO_ROW_WISE) launch(exec_kernel<int32_t, BO_ROW_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<int32_t *>(mem), msize, p);
+        else launch(exec_kernel<int32_t, BO_COLUMN_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<int32_t *>(mem), msize, p);
     }
     return after_launch("exec_kernel");
 }

@@ -25,6 +25,7 @@ __device__ __forceinline__ uint64_t gen_u(uint64_t seed, uint64_t h, uint64_t e)
 
 __global__ void gen_prefix_kernel(uint32_t *dst, long long n, long long p, long long h0, uint64_t seed,
                                   int dtype, int layout, int kind) {
+    pdl_begin();
     const long long total = n * p;
     for (long long idx = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; idx < total;
          idx += static_cast<long long>(gridDim.x) * blockDim.x) {
@@ -50,6 +51,7 @@ __global__ void gen_prefix_kernel(uint32_t *dst, long long n, long long p, long 
 
 __global__ void gen_tri_kernel(uint32_t *dst, long long n, long long p, long long h0, uint64_t seed, int dtype,
                                int layout) {
+    pdl_begin();
     // walks the dense (h, a, b) space; packed layouts store only b - a >= 2
     const long long nn = n * n, total = nn * p;
     for (long long idx = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; idx < total;
@@ -71,6 +73,7 @@ __global__ void gen_tri_kernel(uint32_t *dst, long long n, long long p, long lon
 
 __global__ void checksum_kernel(const uint32_t *v, long long n, long long p, long long h0, int layout,
                                 unsigned long long *acc) {
+    pdl_begin();
     const long long total = n * p;
     uint64_t local = 0;
     for (long long idx = blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x; idx < total;
@@ -94,7 +97,7 @@ static unsigned grid_for(long long total) {
 int launch_gen_prefix(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout, int kind,
                       cudaStream_t st) {
     if (n * p == 0) return BO_OK;
-    gen_prefix_kernel<<<grid_for(n * p), 256, 0, st>>>(static_cast<uint32_t *>(dst), n, p, h0, seed, dtype, layout,
+    launch(gen_prefix_kernel, grid_for(n * p), 256, 0, st, static_cast<uint32_t *>(dst), n, p, h0, seed, dtype, layout,
                                                        kind);
     return after_launch("gen_prefix_kernel");
 }
@@ -102,14 +105,14 @@ int launch_gen_prefix(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed
 int launch_gen_tri(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout,
                    cudaStream_t st) {
     if (n * n * p == 0) return BO_OK;
-    gen_tri_kernel<<<grid_for(n * n * p), 256, 0, st>>>(static_cast<uint32_t *>(dst), n, p, h0, seed, dtype,
+    launch(gen_tri_kernel, grid_for(n * n * p), 256, 0, st, static_cast<uint32_t *>(dst), n, p, h0, seed, dtype,
                                                         layout);
     return after_launch("gen_tri_kernel");
 }
 
 int launch_checksum(const void *v, int64_t n, int64_t p, int64_t h0, int layout, uint64_t *acc, cudaStream_t st) {
     if (n * p == 0) return BO_OK;
-    checksum_kernel<<<grid_for(n * p), 256, 0, st>>>(static_cast<const uint32_t *>(v), n, p, h0, layout,
+    launch(checksum_kernel, grid_for(n * p), 256, 0, st, static_cast<const uint32_t *>(v), n, p, h0, layout,
                                                      reinterpret_cast<unsigned long long *>(acc));
     return after_launch("checksum_kernel");
 }

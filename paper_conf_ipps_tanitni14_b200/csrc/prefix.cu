@@ -41,6 +41,7 @@ __device__ __forceinline__ uint32_t as_bits(T v) {
 template <typename T, int U>
 __global__ void __launch_bounds__(256)
 ps_across_vec4(const T *src, T *dst, long long n, long long p4) {
+    pdl_begin();
     const long long g = blockIdx.x * 256LL + threadIdx.x;
     if (g >= p4) return;
     const uint4 *s = reinterpret_cast<const uint4 *>(src) + g;
@@ -73,6 +74,7 @@ ps_across_vec4(const T *src, T *dst, long long n, long long p4) {
 template <typename T, int U>
 __global__ void __launch_bounds__(256)
 ps_across_scalar(const T *src, T *dst, long long n, long long p) {
+    pdl_begin();
     const long long j = blockIdx.x * 256LL + threadIdx.x;
     if (j >= p) return;
     T r = T(0);
@@ -120,6 +122,7 @@ template <typename T, int kInst>
 __global__ void __launch_bounds__(kInst)
 ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant__ CUtensorMap dst_map,
                  long long ntiles, int nchunks, int slot) {
+    pdl_begin();
     using fr::kElems;
     constexpr int kStages = fr::Cfg<kInst>::kStages;
     constexpr uint32_t kBoxBytes = fr::Cfg<kInst>::kBoxBytes;
@@ -226,6 +229,7 @@ template <typename T, int kInst>
 __global__ void __launch_bounds__(kInst)
 ps_across_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant__ CUtensorMap dst_map,
               long long ntiles, int nchunks, int slot) {
+    pdl_begin();
     using ac::kElems;
     constexpr int kStages = ac::kStages;
     constexpr uint32_t kBoxBytes = ac::Cfg<kInst>::kBoxBytes;
@@ -300,6 +304,7 @@ ps_across_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant
 template <typename T>
 __global__ void __launch_bounds__(128)
 ps_fused_row_smem(const T *src, T *dst, long long n, long long p) {
+    pdl_begin();
     __shared__ T tile[128][33];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     for (long long t0 = blockIdx.x * 128LL; t0 < p; t0 += 128LL * gridDim.x) {
@@ -339,6 +344,7 @@ __device__ __forceinline__ T warp_incl_scan(T x, int lane) {
 template <typename T, bool kVec>
 __global__ void __launch_bounds__(256)
 ps_warpscan(const T *src, T *dst, long long n, long long p) {
+    pdl_begin();
     const int lane = threadIdx.x & 31;
     const long long warps = (static_cast<long long>(gridDim.x) * blockDim.x) >> 5;
     for (long long h = (blockIdx.x * static_cast<long long>(blockDim.x) + threadIdx.x) >> 5; h < p;
@@ -381,6 +387,7 @@ ps_warpscan(const T *src, T *dst, long long n, long long p) {
 template <typename T>
 __global__ void __launch_bounds__(64)
 ps_naive(const T *src, T *dst, long long n, long long p, int layout) {
+    pdl_begin();
     const long long j = blockIdx.x * 64LL + threadIdx.x;
     if (j >= p) return;
     T r = T(0);
@@ -425,7 +432,7 @@ static int launch_across_tma(const T *src, T *dst, int64_t n, int64_t p, cudaStr
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ps_across_tma<T, INST>, INST, C::kSmem);
     const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
     const int slot = fr_next_slot();
-    ps_across_tma<T, INST><<<static_cast<unsigned>(grid), INST, C::kSmem, st>>>(smap, dmap, ntiles, nchunks, slot);
+    launch(ps_across_tma<T, INST>, static_cast<unsigned>(grid), INST, C::kSmem, st, smap, dmap, ntiles, nchunks, slot);
     return after_launch("ps_across_tma");
 }
 
@@ -449,11 +456,11 @@ static int launch_across(const T *src, T *dst, int64_t n, int64_t p, cudaStream_
 #ifndef BO_ACROSS_U
 #define BO_ACROSS_U 8
 #endif
-        ps_across_vec4<T, BO_ACROSS_U><<<grid, 256, 0, st>>>(src, dst, n, p4);
+        launch(ps_across_vec4<T, BO_ACROSS_U>, grid, 256, 0, st, src, dst, n, p4);
         return after_launch("ps_across_vec4");
     }
     const unsigned grid = static_cast<unsigned>((p + 255) / 256);
-    ps_across_scalar<T, 16><<<grid, 256, 0, st>>>(src, dst, n, p);
+    launch(ps_across_scalar<T, 16>, grid, 256, 0, st, src, dst, n, p);
     return after_launch("ps_across_scalar");
 }
 
@@ -472,7 +479,7 @@ static int launch_fused_row_tma(const T *src, T *dst, int64_t n, int64_t p, cuda
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ps_fused_row_tma<T, INST>, INST, C::kSmem);
     const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
     const int slot = fr_next_slot();
-    ps_fused_row_tma<T, INST><<<static_cast<unsigned>(grid), INST, C::kSmem, st>>>(smap, dmap, ntiles, nchunks,
+    launch(ps_fused_row_tma<T, INST>, static_cast<unsigned>(grid), INST, C::kSmem, st, smap, dmap, ntiles, nchunks,
                                                                                    slot);
     return after_launch("ps_fused_row_tma");
 }
@@ -484,7 +491,7 @@ static int launch_fused_row(const T *src, T *dst, int64_t n, int64_t p, cudaStre
         return launch_fused_row_tma<T, 128>(src, dst, n, p, st);
     }
     const long long blocks = std::min<long long>((p + 127) / 128, 16LL * num_sms());
-    ps_fused_row_smem<T><<<static_cast<unsigned>(blocks), 128, 0, st>>>(src, dst, n, p);
+    launch(ps_fused_row_smem<T>, static_cast<unsigned>(blocks), 128, 0, st, src, dst, n, p);
     return after_launch("ps_fused_row_smem");
 }
 
@@ -492,9 +499,9 @@ template <typename T>
 static int launch_warpscan(const T *src, T *dst, int64_t n, int64_t p, cudaStream_t st) {
     const long long blocks = std::min<long long>((p + 7) / 8, 32LL * num_sms());
     if (n % 4 == 0 && aligned16(src) && aligned16(dst))
-        ps_warpscan<T, true><<<static_cast<unsigned>(blocks), 256, 0, st>>>(src, dst, n, p);
+        launch(ps_warpscan<T, true>, static_cast<unsigned>(blocks), 256, 0, st, src, dst, n, p);
     else
-        ps_warpscan<T, false><<<static_cast<unsigned>(blocks), 256, 0, st>>>(src, dst, n, p);
+        launch(ps_warpscan<T, false>, static_cast<unsigned>(blocks), 256, 0, st, src, dst, n, p);
     return after_launch("ps_warpscan");
 }
 
@@ -518,7 +525,7 @@ static int run_prefix(const T *src, T *dst, int64_t n, int64_t p, int layout, in
         }
         case BO_PS_NAIVE: {
             const unsigned grid = static_cast<unsigned>((p + 63) / 64);
-            ps_naive<T><<<grid, 64, 0, st>>>(src, dst, n, p, layout);
+            launch(ps_naive<T>, grid, 64, 0, st, src, dst, n, p, layout);
             return after_launch("ps_naive");
         }
         default:

@@ -35,6 +35,7 @@ __device__ WorkSlot g_tr_slots[kWorkSlots];
 __global__ void __launch_bounds__(tr::kThreads)
 transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
                      const __grid_constant__ CUtensorMap dst_map, int tiles_c, long long ntiles, int slot) {
+    pdl_begin();
     using namespace tr;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *base = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -117,6 +118,7 @@ transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
 __global__ void __launch_bounds__(256)
 transpose_smem_kernel(const uint32_t *__restrict__ src, uint32_t *__restrict__ dst, long long rows,
                       long long cols, long long tiles_c, long long ntiles) {
+    pdl_begin();
     __shared__ uint32_t tile[32][33];
     const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;   // 32 x 8
     for (long long t = blockIdx.x; t < ntiles; t += gridDim.x) {
@@ -158,13 +160,13 @@ int launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, cud
         const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
         static std::atomic<unsigned> next_slot{0};
         const int slot = static_cast<int>(next_slot.fetch_add(1) % kWorkSlots);
-        transpose_tma_kernel<<<static_cast<unsigned>(grid), tr::kThreads, tr::kSmem, st>>>(
+        launch(transpose_tma_kernel, static_cast<unsigned>(grid), tr::kThreads, tr::kSmem, st, 
             smap, dmap, static_cast<int>(tiles_c), ntiles, slot);
         return after_launch("transpose_tma_kernel");
     }
     const long long tiles_c = (cols + 31) / 32, ntiles = tiles_c * ((rows + 31) / 32);
     const long long grid = std::min<long long>(ntiles, 16LL * num_sms());
-    transpose_smem_kernel<<<static_cast<unsigned>(grid), 256, 0, st>>>(
+    launch(transpose_smem_kernel, static_cast<unsigned>(grid), 256, 0, st, 
         static_cast<const uint32_t *>(src), static_cast<uint32_t *>(dst), rows, cols, tiles_c, ntiles);
     return after_launch("transpose_smem_kernel");
 }

@@ -57,6 +57,7 @@ __host__ __device__ __forceinline__ long long c_index(int layout, long long h, l
 template <typename T, int N, int LAYOUT>   // layout a template parameter: the 105+ weight
 __global__ void __launch_bounds__(128)      // loads must be branch-free so they issue early
 tri_thread_reg(const T *__restrict__ c, T *__restrict__ out, long long p) {
+    pdl_begin();
     constexpr int layout = LAYOUT;
     using Op = MinPlus<T>;
     const long long h = blockIdx.x * 128LL + threadIdx.x;
@@ -91,6 +92,7 @@ tri_thread_reg(const T *__restrict__ c, T *__restrict__ out, long long p) {
 template <typename T, int N, int LAYOUT, int S, int W>
 __global__ void __launch_bounds__(32 * W)
 tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out, long long p, long long nbatch) {
+    pdl_begin();
     using Op = MinPlus<T>;
     constexpr int NE = LAYOUT == BO_PACKED_ROW ? (N - 1) * (N - 2) / 2   // packed: every weight is read
                                                : (N - 3) * N + N;        // c[N-3][N-1] is the last one read
@@ -180,6 +182,7 @@ __device__ __forceinline__ void bulk_load_1d(void *dst, const void *src, uint32_
 template <typename T, int N>
 __global__ void __launch_bounds__(32)
 tri_thread_reg_packed(const T *__restrict__ c, T *__restrict__ out, long long p, long long nbatch) {
+    pdl_begin();
     using Op = MinPlus<T>;
     constexpr int K = (N - 1) * (N - 2) / 2;
     constexpr uint32_t kBatchBytes = 32u * K * sizeof(T);
@@ -237,6 +240,7 @@ tri_thread_reg_packed(const T *__restrict__ c, T *__restrict__ out, long long p,
 template <typename T>
 __global__ void __launch_bounds__(64)
 tri_umm_global(const T *__restrict__ c, T *__restrict__ out, T *M, long long n, long long p, int layout) {
+    pdl_begin();
     const long long h = blockIdx.x * 64LL + threadIdx.x;
     if (h >= p) return;
     const long long n1 = n - 1;
@@ -264,6 +268,7 @@ tri_umm_global(const T *__restrict__ c, T *__restrict__ out, T *M, long long n, 
 template <typename T>
 __global__ void __launch_bounds__(512)
 tri_smem_warp(const T *__restrict__ c, T *__restrict__ out, int n, long long p, int layout, int SP, int W) {
+    pdl_begin();
     using Op = MinPlus<T>;
     extern __shared__ uint8_t smem_raw[];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -378,7 +383,7 @@ static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) 
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * W, smem);
     // enough CTAs that every warp of every resident CTA has a batch
     const long long grid = std::min<long long>((nbatch + W - 1) / W, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
-    kern<<<static_cast<unsigned>(grid), 32 * W, smem, st>>>(map, static_cast<T *>(out), p, nbatch);
+    launch(kern, static_cast<unsigned>(grid), 32 * W, smem, st, map, static_cast<T *>(out), p, nbatch);
     return after_launch("tri_thread_reg_tma");
 }
 
@@ -393,7 +398,7 @@ static int launch_reg_packed(const void *c, void *out, int64_t p, cudaStream_t s
     int per_sm = 1;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_thread_reg_packed<T, N>, 32, smem);
     const long long grid = std::min<long long>(nbatch, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
-    tri_thread_reg_packed<T, N><<<static_cast<unsigned>(grid), 32, smem, st>>>(
+    launch(tri_thread_reg_packed<T, N>, static_cast<unsigned>(grid), 32, smem, st, 
         static_cast<const T *>(c), static_cast<T *>(out), p, nbatch);
     return after_launch("tri_thread_reg_packed");
 }
@@ -409,10 +414,10 @@ static int launch_reg_n(const void *c, void *out, int64_t p, int layout, cudaStr
     const T *cc = static_cast<const T *>(c);
     T *oo = static_cast<T *>(out);
     switch (layout) {
-        case BO_ROW_WISE: tri_thread_reg<T, N, BO_ROW_WISE><<<grid, 128, 0, st>>>(cc, oo, p); break;
-        case BO_COLUMN_WISE: tri_thread_reg<T, N, BO_COLUMN_WISE><<<grid, 128, 0, st>>>(cc, oo, p); break;
-        case BO_PACKED_ROW: tri_thread_reg<T, N, BO_PACKED_ROW><<<grid, 128, 0, st>>>(cc, oo, p); break;
-        default: tri_thread_reg<T, N, BO_PACKED_COLUMN><<<grid, 128, 0, st>>>(cc, oo, p); break;
+        case BO_ROW_WISE: launch(tri_thread_reg<T, N, BO_ROW_WISE>, grid, 128, 0, st, cc, oo, p); break;
+        case BO_COLUMN_WISE: launch(tri_thread_reg<T, N, BO_COLUMN_WISE>, grid, 128, 0, st, cc, oo, p); break;
+        case BO_PACKED_ROW: launch(tri_thread_reg<T, N, BO_PACKED_ROW>, grid, 128, 0, st, cc, oo, p); break;
+        default: launch(tri_thread_reg<T, N, BO_PACKED_COLUMN>, grid, 128, 0, st, cc, oo, p); break;
     }
     return after_launch("tri_thread_reg");
 }
@@ -445,7 +450,7 @@ static int launch_smem_warp(const void *c, void *out, int64_t n, int64_t p, int 
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_smem_warp<T>, W * 32, smem);
     per_sm = std::max(per_sm, 1);
     const long long blocks = std::min<long long>((p + W - 1) / W, static_cast<long long>(per_sm) * num_sms() * 8);
-    tri_smem_warp<T><<<static_cast<unsigned>(blocks), W * 32, smem, st>>>(
+    launch(tri_smem_warp<T>, static_cast<unsigned>(blocks), W * 32, smem, st, 
         static_cast<const T *>(c), static_cast<T *>(out), static_cast<int>(n), p, layout, smem_sp(n), W);
     return after_launch("tri_smem_warp");
 }
@@ -458,7 +463,7 @@ static int run_tri(const void *c, void *out, int64_t n, int64_t p, int layout, i
             return launch_reg<T>(c, out, n, p, layout, st);
         case BO_TRI_UMM_GLOBAL: {
             const unsigned grid = static_cast<unsigned>((p + 63) / 64);
-            tri_umm_global<T><<<grid, 64, 0, st>>>(static_cast<const T *>(c), static_cast<T *>(out),
+            launch(tri_umm_global<T>, grid, 64, 0, st, static_cast<const T *>(c), static_cast<T *>(out),
                                                    static_cast<T *>(ws), n, p, layout);
             return after_launch("tri_umm_global");
         }

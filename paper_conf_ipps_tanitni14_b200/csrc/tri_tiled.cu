@@ -518,6 +518,7 @@ template <typename T, int LPI, bool CHORDS>
 __global__ void __launch_bounds__(128, 1)
 tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restrict__ chords, int n, long long p,
                  int layout, int NT, int c_vec, uint64_t lsched) {
+    pdl_begin();
     using Op = tt::Ops<T>;
     using T4 = typename tt::V4<T>::type;
     using tt::xc;
@@ -728,7 +729,7 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
     const long long blocks = std::min<long long>((p + per_cta - 1) / per_cta,
                                                  static_cast<long long>(per_sm) * num_sms());
     const int c_vec = (n % 4 == 0) && aligned16(c);
-    tri_tiled_kernel<T, LPI, CHORDS><<<static_cast<unsigned>(blocks), W * 32, smem, st>>>(
+    launch(tri_tiled_kernel<T, LPI, CHORDS>, static_cast<unsigned>(blocks), W * 32, smem, st, 
         static_cast<const T *>(c), static_cast<T *>(out), chords, static_cast<int>(n), p, layout, NT, c_vec,
         split_schedule(NT, LPI));
     return after_launch("tri_tiled_kernel");
@@ -770,6 +771,7 @@ template <typename T>
 __global__ void __launch_bounds__(512, 1)
 tri_tiled_global_kernel(const T *__restrict__ c, T *__restrict__ out, T *ws, int n, long long p, int layout, int NT,
                         int c_vec) {
+    pdl_begin();
     using Op = tt::Ops<T>;
     using T4 = typename tt::V4<T>::type;
     using tt::xc;
@@ -873,11 +875,11 @@ int launch_tri_tiled_global(const void *c, void *out, void *ws, int64_t n, int64
     const int threads = tiled_global_threads(n);
     const int c_vec = (n % 4 == 0) && aligned16(c);
     if (dtype == BO_F32)
-        tri_tiled_global_kernel<float><<<static_cast<unsigned>(grid), threads, 0, st>>>(
+        launch(tri_tiled_global_kernel<float>, static_cast<unsigned>(grid), threads, 0, st, 
             static_cast<const float *>(c), static_cast<float *>(out), static_cast<float *>(ws), static_cast<int>(n), p,
             layout, NT, c_vec);
     else
-        tri_tiled_global_kernel<int32_t><<<static_cast<unsigned>(grid), threads, 0, st>>>(
+        launch(tri_tiled_global_kernel<int32_t>, static_cast<unsigned>(grid), threads, 0, st, 
             static_cast<const int32_t *>(c), static_cast<int32_t *>(out), static_cast<int32_t *>(ws),
             static_cast<int>(n), p, layout, NT, c_vec);
     return after_launch("tri_tiled_global_kernel");
