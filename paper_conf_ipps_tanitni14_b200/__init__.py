@@ -220,14 +220,20 @@ def triangulation(c: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, 
     return out
 
 
-def triangulation_chords(c: torch.Tensor, layout: int = ROW_WISE, stream=None):
+def triangulation_chords(c: torch.Tensor, layout: int = ROW_WISE, stream=None, out: torch.Tensor | None = None,
+                         chords: torch.Tensor | None = None):
     """Values and the chords of an optimal triangulation (NEXT-1):
     returns (out [p], chords [p, n-3, 2] int16 vertex pairs)."""
     _need_cuda(c)
     n, p = _tri_shape(c, layout)
     dt = _dtype_code(c)
-    out = torch.empty(p, dtype=c.dtype, device=c.device)
-    chords = torch.empty((p, max(n - 3, 0), 2), dtype=torch.int16, device=c.device)
+    if out is None:
+        out = torch.empty(p, dtype=c.dtype, device=c.device)
+    if chords is None:
+        chords = torch.empty((p, max(n - 3, 0), 2), dtype=torch.int16, device=c.device)
+    _need_cuda(out, chords)
+    if out.dtype != c.dtype or out.numel() != p or chords.dtype != torch.int16 or chords.numel() != p * max(n - 3, 0) * 2:
+        raise ValueError("out must be [p] of the weights' dtype and chords [p, n-3, 2] int16")
     _check(lib().bulk_triangulation_chords(c.data_ptr(), out.data_ptr(), chords.data_ptr() if chords.numel() else None,
                                            n, p, dt, layout, _stream(stream)))
     return out, chords
