@@ -31,18 +31,17 @@ inline int after_launch(const char *what) {
 
 // Programmatic dependent launch (PDL).  Every kernel is launched with
 // cudaLaunchAttributeProgrammaticStreamSerialization and begins with
-// pdl_begin(): it lets the next kernel in the stream launch as soon as all of
-// its own CTAs have started (griddepcontrol.launch_dependents) and waits for
-// the previous kernel to complete and its memory to be visible
-// (griddepcontrol.wait) before it touches global memory.  Stream order is
-// kept -- nothing is read or written before the predecessor has finished --
-// but launch latency and the predecessor's tail overlap (measured on B200,
-// tools/micro/pdl_gap.cu: a 128 KB kernel 3.5 -> 1.2 us per launch back to
-// back, a 16 MB one 8.2 -> 5.7 us).  Without the attribute both are no-ops.
-__device__ __forceinline__ void pdl_begin() {
-    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-    asm volatile("griddepcontrol.wait;" ::: "memory");
-}
+// pdl_begin() = griddepcontrol.wait: it waits for the previous kernel in the
+// stream to complete and its memory to be visible before it touches global
+// memory, so stream order is kept, but the launch itself is processed while
+// the predecessor drains (measured on B200, tools/micro/pdl_gap.cu: a 128 KB
+// kernel 3.5 -> 1.2 us per launch back to back, a 16 MB one 8.2 -> 5.7 us).
+// No kernel calls griddepcontrol.launch_dependents early: the implicit trigger
+// at exit keeps the successor's CTAs off SMs the predecessor still occupies
+// (an early trigger packed a small successor grid onto the few idle SMs:
+// 1024 64-gons 17 -> 23 us; tools/micro/pdl_place.cu: the implicit trigger
+// keeps ~90 % of the gain).  Without the attribute the wait is a no-op.
+__device__ __forceinline__ void pdl_begin() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 template <typename... KArgs, typename... Args>
 inline void launch(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args &&...args) {
     cudaLaunchAttribute at[1];
