@@ -27,11 +27,13 @@ AUTO = 0
 PS_ACROSS, PS_WARPSCAN, PS_FUSED_ROW, PS_TRANSPOSED, PS_NAIVE = 1, 2, 3, 4, 5
 TRI_UMM_GLOBAL, TRI_SMEM_WARP, TRI_THREAD_REG, TRI_TILED, TRI_TILED_HALF, TRI_TILED_GLOBAL = 16, 17, 18, 19, 20, 21
 TRI_TILED_QUARTER = 22
+TRI_TILED_GLOBAL8 = 23
 VARIANT_NAMES = {
     AUTO: "auto", PS_ACROSS: "across", PS_WARPSCAN: "warpscan", PS_FUSED_ROW: "fused_row",
     PS_TRANSPOSED: "transposed", PS_NAIVE: "naive", TRI_UMM_GLOBAL: "umm_global",
     TRI_SMEM_WARP: "smem_warp", TRI_THREAD_REG: "thread_reg", TRI_TILED: "tiled", TRI_TILED_HALF: "tiled_half",
     TRI_TILED_GLOBAL: "tiled_global", TRI_TILED_QUARTER: "tiled_quarter",
+    TRI_TILED_GLOBAL8: "tiled_global8",
 }
 KINDS = {"uniform": 0, "ones": 1, "arange": 2, "smallint": 3}
 

@@ -132,7 +132,7 @@ static int check_tri_args(const void *c, const void *out, int64_t n, int64_t p, 
     if (!valid_tri_layout(layout)) return fail(BO_EINVAL, "triangulation: bad layout");
     if (p > kMaxElems / (n * n)) return fail(BO_EINVAL, "triangulation: n*n*p too large");
     if (p > 0 && (!c || !out)) return fail(BO_EINVAL, "triangulation: NULL pointer");
-    if (variant != BO_AUTO && (variant < BO_TRI_UMM_GLOBAL || variant > BO_TRI_TILED_QUARTER))
+    if (variant != BO_AUTO && (variant < BO_TRI_UMM_GLOBAL || variant > BO_TRI_TILED_GLOBAL8))
         return fail(BO_EINVAL, "triangulation: unknown variant");
     return BO_OK;
 }
@@ -381,14 +381,15 @@ int bulk_prefix_sums_host(const void *h_src, void *h_dst, int64_t n, int64_t p, 
 // the chunks use disjoint slices of one p-sized workspace; TILED_GLOBAL keeps
 // a table per CTA, so each of the two streams gets its own chunk-sized copy.
 static size_t tri_host_ws(int64_t n, int64_t p, int v) {
-    if (v == BO_TRI_TILED_GLOBAL) return 2 * tri_workspace(n, host_chunk(p), v);
+    if (v == BO_TRI_TILED_GLOBAL || v == BO_TRI_TILED_GLOBAL8) return 2 * tri_workspace(n, host_chunk(p), v);
     return tri_workspace(n, p, v);
 }
 
 size_t bulk_triangulation_host_bytes(int64_t n, int64_t p, int dtype, int layout, int variant) {
     if (n < 3 || p <= 0 || !valid_tri_layout(layout)) return 0;
     const int v = resolve_tri_variant(n, p, dtype, layout, variant);
-    return static_cast<size_t>(tri_words(n, layout)) * p * 4 + static_cast<size_t>(p) * 4 + tri_host_ws(n, p, v);
+    const size_t ws_off = (static_cast<size_t>(tri_words(n, layout)) * p * 4 + static_cast<size_t>(p) * 4 + 255) & ~size_t(255);
+    return ws_off + tri_host_ws(n, p, v);
 }
 
 int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, int dtype, int layout,
@@ -402,9 +403,10 @@ int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, 
     const size_t nn = static_cast<size_t>(tri_words(n, layout));     // weights per instance
     const size_t c_bytes = nn * p * 4, out_bytes = static_cast<size_t>(p) * 4;
     const size_t ws_bytes = tri_host_ws(n, p, v);
-    if (!d_buf || d_bytes < c_bytes + out_bytes + ws_bytes)
+    const size_t ws_off = (c_bytes + out_bytes + 255) & ~size_t(255);   // workspace 256-byte aligned
+    if (!d_buf || d_bytes < ws_off + ws_bytes)
         return fail(BO_EINVAL, "triangulation_host: device buffer too small (need " +
-                                   std::to_string(c_bytes + out_bytes + ws_bytes) + " bytes)");
+                                   std::to_string(ws_off + ws_bytes) + " bytes)");
     HostPipe *hp = host_pipe();
     cudaStream_t caller = static_cast<cudaStream_t>(stream);
     if ((rc = cuda_check(cudaEventRecord(hp->ev_start, caller), "tri_host: event"))) return rc;
@@ -414,7 +416,7 @@ int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, 
     char *ho = static_cast<char *>(h_out);
     char *db = static_cast<char *>(d_buf);
     char *dout = db + c_bytes;
-    char *dws = db + c_bytes + out_bytes;
+    char *dws = db + ws_off;
     int k = 0;
     for (int64_t p0 = 0; p0 < p; p0 += ch, ++k) {
         const int64_t pc = std::min(ch, p - p0);

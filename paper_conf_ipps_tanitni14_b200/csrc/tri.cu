@@ -331,6 +331,9 @@ int launch_tri_tiled_global(const void *c, void *out, void *ws, int64_t n, int64
                             cudaStream_t st);
 int launch_tri_tiled(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout, int lpi,
                      cudaStream_t st);
+size_t tiled_global8_workspace(int64_t n, int64_t p);
+int launch_tri_global8(const void *c, void *out, void *ws, int64_t n, int64_t p, int dtype, int layout,
+                       cudaStream_t st);
 
 static int smem_sp(int64_t n) {
     const int n1 = static_cast<int>(n - 1);
@@ -346,12 +349,13 @@ int resolve_tri_variant(int64_t n, int64_t p, int dtype, int layout, int variant
     // 8 lanes per instance (two tiles per lane on the long tile-diagonals) up to
     // n = 56 (1.1-1.6x faster than 16 lanes, tools/tri_time.py --cmp); 16 lanes above
     if (tiled_supported(n)) return n <= 56 ? BO_TRI_TILED_QUARTER : BO_TRI_TILED_HALF;
-    return BO_TRI_TILED_GLOBAL;
+    return n >= 512 ? BO_TRI_TILED_GLOBAL8 : BO_TRI_TILED_GLOBAL;   // 8x8 tiles pay from n ~ 450 (tri_global8.cu)
 }
 
 size_t tri_workspace(int64_t n, int64_t p, int variant) {
     if (variant == BO_TRI_UMM_GLOBAL) return static_cast<size_t>(n - 1) * (n - 1) * p * 4;
     if (variant == BO_TRI_TILED_GLOBAL) return tiled_global_workspace(n, p);
+    if (variant == BO_TRI_TILED_GLOBAL8) return tiled_global8_workspace(n, p);
     return 0;
 }
 
@@ -478,6 +482,8 @@ static int run_tri(const void *c, void *out, int64_t n, int64_t p, int layout, i
         case BO_TRI_TILED_GLOBAL:
             return launch_tri_tiled_global(c, out, ws, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout,
                                            st);
+        case BO_TRI_TILED_GLOBAL8:
+            return launch_tri_global8(c, out, ws, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout, st);
         default:
             return fail(BO_EINVAL, "triangulation: unknown variant");
     }

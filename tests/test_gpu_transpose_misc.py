@@ -103,7 +103,7 @@ def test_launch_counter_counts_kernels():
 
 
 @pytest.mark.parametrize("n,p,variant", [(40, 1500, bo.AUTO), (40, 1500, bo.TRI_TILED_HALF),
-                                         (80, 600, bo.TRI_TILED_GLOBAL), (16, 700, bo.TRI_THREAD_REG)])
+                                         (80, 600, bo.TRI_TILED_GLOBAL), (80, 333, bo.TRI_TILED_GLOBAL8), (16, 700, bo.TRI_THREAD_REG)])
 @pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
 def test_tri_host_entry_point_chunked_variants(n, p, variant, layout):
     # several chunks in flight on the two internal streams; TILED_GLOBAL gives each stream its own scratch

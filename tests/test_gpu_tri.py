@@ -18,7 +18,7 @@ NTHREADS = os.cpu_count() or 1
 
 
 def _variants(n):
-    v = [bo.AUTO, bo.TRI_UMM_GLOBAL, bo.TRI_SMEM_WARP, bo.TRI_TILED_GLOBAL]
+    v = [bo.AUTO, bo.TRI_UMM_GLOBAL, bo.TRI_SMEM_WARP, bo.TRI_TILED_GLOBAL, bo.TRI_TILED_GLOBAL8]
     if n <= 18:
         v.append(bo.TRI_THREAD_REG)
     if 5 <= n <= 64:
@@ -104,7 +104,7 @@ def test_tr2_full_config(layout):
 
 
 @pytest.mark.parametrize("variant", [bo.TRI_SMEM_WARP, bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_TILED_QUARTER,
-                                     bo.TRI_TILED_GLOBAL, bo.TRI_UMM_GLOBAL])
+                                     bo.TRI_TILED_GLOBAL, bo.TRI_TILED_GLOBAL8, bo.TRI_UMM_GLOBAL])
 def test_tr2_variants_agree_full_size(variant):
     n, p = 64, 65536
     c = bo.generate_tri(n, p, 4, torch.float32, bo.ROW_WISE)
@@ -158,11 +158,22 @@ def test_chords_tr2_full_size_sampled():
 # ------------------------------------------------ NEXT-2: the paper's large polygons
 @pytest.mark.parametrize("dt", ["int32", "float32"])
 @pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
-@pytest.mark.parametrize("n,p", [(256, 5), (512, 3), (130, 20)])
-def test_large_polygons_match_oracle(dt, layout, n, p):
+@pytest.mark.parametrize("n,p", [(256, 5), (512, 3), (130, 20), (203, 7)])
+@pytest.mark.parametrize("variant", [bo.AUTO, bo.TRI_TILED_GLOBAL, bo.TRI_TILED_GLOBAL8])
+def test_large_polygons_match_oracle(dt, layout, n, p, variant):
     c = bulkgen.tri_input(n, p, seed=n + p, dtype=dt, layout=layout)
     ref = oracle.bulk_opt(c, layout, nthreads=NTHREADS)
-    got = bo.triangulation(torch.from_numpy(c).to(DEV), layout).cpu().numpy()       # AUTO -> TILED_GLOBAL
+    got = bo.triangulation(torch.from_numpy(c).to(DEV), layout, variant).cpu().numpy()
+    assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+
+
+def test_global8_many_instances_per_cta():
+    # p > #SMs: every CTA reuses its table slot for several instances (stale cells from the
+    # previous instance must not leak into the next one)
+    n, p = 72, 700
+    c = bulkgen.tri_input(n, p, seed=11, dtype="float32")
+    ref = oracle.bulk_opt(c, oracle.ROW_WISE, nthreads=NTHREADS)
+    got = bo.triangulation(torch.from_numpy(c).to(DEV), bo.ROW_WISE, bo.TRI_TILED_GLOBAL8).cpu().numpy()
     assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
 
 

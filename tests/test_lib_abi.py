@@ -99,6 +99,7 @@ def test_workspace_and_variant_queries(L):
     assert bo.triangulation_variant(64, 100, bo.F32, bo.ROW_WISE) == bo.TRI_TILED_HALF
     assert bo.triangulation_variant(40, 100, bo.F32, bo.ROW_WISE) == bo.TRI_TILED_QUARTER
     assert bo.triangulation_variant(100, 100, bo.F32, bo.ROW_WISE) == bo.TRI_TILED_GLOBAL
+    assert bo.triangulation_variant(512, 100, bo.F32, bo.ROW_WISE) == bo.TRI_TILED_GLOBAL8
 
 
 def test_binding_refuses_cpu_tensors(L):
