@@ -30,6 +30,9 @@ for layout in (bo.PACKED_ROW, bo.PACKED_COLUMN):
         bo.triangulation_chords(c, layout)
 c = bo.generate_tri(80, 3, 1, torch.float32, bo.ROW_WISE)
 bo.triangulation(c, bo.ROW_WISE, bo.TRI_TILED_GLOBAL)
+bo.triangulation(c, bo.ROW_WISE, bo.TRI_TILED_GLOBAL8)
+for layout in (bo.COLUMN_WISE, bo.PACKED_ROW):
+    bo.triangulation(bo.generate_tri(37, 5, 1, torch.int32, layout), layout, bo.TRI_TILED_GLOBAL8)
 from paper_conf_ipps_tanitni14_b200 import programs  # noqa: E402
 for layout in (bo.ROW_WISE, bo.COLUMN_WISE):
     m = bo.generate_prefix(16, 70, 1, torch.float32, layout)
