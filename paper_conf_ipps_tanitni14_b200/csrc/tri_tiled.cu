@@ -194,18 +194,14 @@ __device__ __forceinline__ float2 add2b(float a, float x, float y) {
 }
 __device__ __forceinline__ float min3(float a, float b, float c) { return fminf(fminf(a, b), c); }
 // fp32, row-ordered: P1 terms of a row pair two v's in one FADD2 (A[u][w]
-// broadcast), P3 terms pair v = 2, 3, and mins fold two terms per FMNMX3: 64
-// instructions per tile instead of 112.  (A latency-ordered variant -- cells by
-// anti-diagonal, newest terms last, scalar adds -- measured 5% slower: the
-// kernel is bound by issue slots more than by this chain.)
-#ifndef BO_TRI_FIXZERO
-#define BO_TRI_FIXZERO 1
-#endif
-#if BO_TRI_FIXZERO
-// Same, using that the polygon edges X[a][a+1] of the diagonal tiles are 0
-// (M[i][i] = 0): A[u][u+1] = Bd[w][w+1] = 0, so those terms are
-// t itself (x + 0 == x exactly for the finite, non-negative values of the
-// table, G16) -- 14 instructions less per tile, and Bd rows 2..3 are never read.
+// broadcast), mins fold two terms per FMNMX3, and the polygon edges X[a][a+1]
+// of the diagonal tiles are 0 (M[i][i] = 0): A[u][u+1] =
+// Bd[w][w+1] = 0, so those terms are t itself (x + 0 == x exactly for the
+// finite, non-negative values of the table, G16) -- 14 instructions less per
+// tile than the plain pairing, and Bd rows 2..3 are never read.  (A
+// latency-ordered variant -- cells by anti-diagonal, newest terms last,
+// scalar adds -- measured 5% slower: the kernel is bound by issue slots more
+// than by this chain.)
 template <>
 __device__ __forceinline__ void fixup<float>(float (&t)[4][4], const float (&S)[4][4], const float (&A)[4][4],
                                              const float (&Bd)[4][4], const float (&C)[4][4], bool edge) {
@@ -244,36 +240,6 @@ __device__ __forceinline__ void fixup<float>(float (&t)[4][4], const float (&S)[
     }
     p3(0);
 }
-#else
-template <>
-__device__ __forceinline__ void fixup<float>(float (&t)[4][4], const float (&S)[4][4], const float (&A)[4][4],
-                                             const float (&Bd)[4][4], const float (&C)[4][4], bool edge) {
-#pragma unroll
-    for (int u = 3; u >= 0; --u) {
-        float R[4] = {S[u][0], S[u][1], S[u][2], S[u][3]};
-#pragma unroll
-        for (int w = u + 1; w < 4; w += 2) {                  // P1, two w per FMNMX3
-            const float2 x01 = add2b(A[u][w], t[w][0], t[w][1]), x23 = add2b(A[u][w], t[w][2], t[w][3]);
-            if (w + 1 < 4) {
-                const float2 y01 = add2b(A[u][w + 1], t[w + 1][0], t[w + 1][1]);
-                const float2 y23 = add2b(A[u][w + 1], t[w + 1][2], t[w + 1][3]);
-                R[0] = min3(R[0], x01.x, y01.x); R[1] = min3(R[1], x01.y, y01.y);
-                R[2] = min3(R[2], x23.x, y23.x); R[3] = min3(R[3], x23.y, y23.y);
-            } else {
-                R[0] = fminf(R[0], x01.x); R[1] = fminf(R[1], x01.y);
-                R[2] = fminf(R[2], x23.x); R[3] = fminf(R[3], x23.y);
-            }
-        }
-        // P3, sequential in v
-        t[u][0] = edge && u == 3 ? 0.0f : __fadd_rn(R[0], C[u][0]);
-        const float2 a23 = add2b(t[u][0], Bd[0][2], Bd[0][3]);
-        t[u][1] = __fadd_rn(fminf(R[1], __fadd_rn(t[u][0], Bd[0][1])), C[u][1]);
-        const float2 b23 = add2b(t[u][1], Bd[1][2], Bd[1][3]);
-        t[u][2] = __fadd_rn(min3(R[2], a23.x, b23.x), C[u][2]);
-        t[u][3] = __fadd_rn(min3(fminf(R[3], a23.y), b23.y, __fadd_rn(t[u][2], Bd[2][3])), C[u][3]);
-    }
-}
-#endif
 
 // Dense part of tile (I, J) over chunk-columns m, m + s, ... < J (m < J):
 // software-pipelined ping-pong (load chunk m+s while computing chunk m); the
