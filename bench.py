@@ -48,6 +48,9 @@ WORKLOADS = {
                    desc="bulk prefix-sums fp32 n=1024, p=2^20 per GPU, column-wise resident"),
     "ps2tr": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=4,
                   desc="bulk prefix-sums fp32 n=1024, p=2^20, row-wise via explicit transpose kernels"),
+    "tr_transpose": dict(seed=2, algo="transpose", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=0,
+                         desc="SURVEY row a1: layout transpose of the PS-2 data, row-wise [p][n] -> column-wise "
+                              "[n][p] (P:120-126)"),
     "ps2naive_col": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=1, variant=5,
                          desc="the paper's column-wise kernel (thread per instance, 32-bit accesses)"),
     "ps1": dict(seed=1, algo="prefix", n=32, p=1024, dtype="int32", layout=0, variant=0,
@@ -77,7 +80,7 @@ WORKLOADS = {
     "ps2naive_row": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=5,
                          desc="the paper's row-wise kernel (thread per instance, uncoalesced)"),
 }
-EXTRAS = ["ps2col", "ps2tr", "ps1", "tr1", "tr1col", "tr1packed", "tr2", "tr2packed", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
+EXTRAS = ["ps2col", "ps2tr", "tr_transpose", "ps1", "tr1", "tr1col", "tr1packed", "tr2", "tr2packed", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
           "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col"]
 L2_BYTES = 126 * 2 ** 20
 
@@ -91,7 +94,7 @@ def algo_bytes_per_instance(wl):
     """Algorithmic HBM bytes per instance: prefix reads
     and writes n elements; OPT reads the C(n-1,2) weights c[a][b], b-a>=2
     (the only ones Algorithm OPT touches) and writes one result."""
-    if wl["algo"] in ("prefix", "exec"):
+    if wl["algo"] in ("prefix", "exec", "transpose"):
         return 2 * wl["n"] * 4
     n = wl["n"]
     return 4 * ((n - 1) * (n - 2) // 2 + 1)
@@ -284,6 +287,14 @@ def setup_workload(wl, rank, copies=1):
             bo.execute(prog, nxt(), wl["layout"], prog_buf=pbuf)
         return dict(x=x, out=x, fn=fn, seed=seed, h0=h0,
                     variant=f"exec[{wl['prog']}: {prog.array().shape[0]} instr]")
+    if wl["algo"] == "transpose":
+        x = bo.generate_prefix(n, p, seed, dt, bo.ROW_WISE, "uniform", h0=h0)        # [p][n]
+        out = torch.empty((n, p), dtype=dt, device="cuda")
+        nxt = _rotator(x, copies)
+
+        def fn():
+            bo.transpose(nxt(), out=out)
+        return dict(x=x, out=out, fn=fn, seed=seed, h0=h0, variant="transpose_tma")
     if wl["algo"] == "prefix":
         x = bo.generate_prefix(n, p, seed, dt, wl["layout"], "uniform", h0=h0)
         out = torch.empty_like(x)
@@ -319,7 +330,7 @@ def setup_workload(wl, rank, copies=1):
 
 def input_bytes(wl):
     n, p = wl["n"], wl["p"]
-    if wl["algo"] in ("prefix", "exec"):
+    if wl["algo"] in ("prefix", "exec", "transpose"):
         return n * p * 4
     return ((n - 1) * (n - 2) // 2 if wl["layout"] >= 2 else n * n) * p * 4
 
@@ -336,11 +347,11 @@ def measure(ctx, name, steps, warmup, stream, peaks, traffic):
            "l2": l2_note(wl, copies),
            "gpu_launches": launches}
     bytes_launch = algo_bytes_per_instance(wl) * wl["p"]
-    if wl["algo"] in ("prefix", "exec"):
+    if wl["algo"] in ("prefix", "exec", "transpose"):
         gbs = bytes_launch / (ms * 1e-3) / 1e9
         res["algorithmic_GBps_per_gpu"] = gbs
         res["roofline"] = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                           "frac": gbs / peaks["hbm_gbs"]}
+                           "frac": gbs / peaks["hbm_gbs"], "traffic": traffic.get(name, {}).get("dram_bytes_per_launch")}
     else:
         res["roofline"] = tri_roofline(wl, ms * steps / max(1, launches), peaks)
     return res, st
@@ -653,7 +664,7 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--workload", default="ps2", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default="ps2", choices=sorted(k for k in WORKLOADS if WORKLOADS[k]["algo"] != "transpose"))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-extras", dest="extras", action="store_false")
     ap.add_argument("--no-e2e", dest="e2e", action="store_false")
