@@ -1,0 +1,70 @@
+"""GPU: the library on user streams.  Kernels with dynamic tile queues
+(fused-row / column-wise prefix, transpose) draw a queue slot per launch, and
+every kernel is launched with programmatic dependent launch (griddepcontrol.wait
+before any global access): launches in flight on several streams at once, and
+chains of dependent launches with no host synchronisation in between, must give
+exactly the results of one launch at a time."""
+import numpy as np
+import pytest
+import torch
+
+import bulkgen
+import oracle
+import paper_conf_ipps_tanitni14_b200 as bo
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda"
+
+
+def test_concurrent_streams_match_serial():
+    n, p = 1024, 40000                       # the 128-instance TMA fused-row kernel, dynamic queue
+    xs = [bo.generate_prefix(n, p, 20 + k, torch.float32, bo.ROW_WISE) for k in range(6)]
+    ref = [bo.prefix_sums(x, bo.ROW_WISE) for x in xs]
+    torch.cuda.synchronize()
+    streams = [torch.cuda.Stream() for _ in range(3)]
+    outs = [torch.empty_like(x) for x in xs]
+    for rep in range(3):
+        for k, x in enumerate(xs):
+            s = streams[k % len(streams)]
+            with torch.cuda.stream(s):
+                bo.prefix_sums(x, bo.ROW_WISE, out=outs[k], stream=s)
+        torch.cuda.synchronize()
+        for k in range(len(xs)):
+            assert torch.equal(outs[k].view(torch.int32), ref[k].view(torch.int32)), (rep, k)
+
+
+def test_concurrent_triangulation_with_workspace():
+    # TILED_GLOBAL keeps a table per CTA in the caller's workspace: one workspace per stream
+    n, p = 80, 300
+    cs = [bo.generate_tri(n, p, 30 + k, torch.float32, bo.ROW_WISE) for k in range(4)]
+    ref = [bo.triangulation(c, bo.ROW_WISE, bo.TRI_TILED_GLOBAL) for c in cs]
+    torch.cuda.synchronize()
+    streams = [torch.cuda.Stream() for _ in range(2)]
+    need = bo.triangulation_workspace(n, p, bo.F32, bo.ROW_WISE, bo.TRI_TILED_GLOBAL)
+    wss = [torch.empty(need, dtype=torch.uint8, device=DEV) for _ in streams]
+    outs = [torch.empty(p, dtype=torch.float32, device=DEV) for _ in cs]
+    for k, c in enumerate(cs):
+        s = streams[k % 2]
+        bo.triangulation(c, bo.ROW_WISE, bo.TRI_TILED_GLOBAL, out=outs[k], workspace=wss[k % 2], stream=s)
+    torch.cuda.synchronize()
+    for k in range(len(cs)):
+        assert torch.equal(outs[k].view(torch.int32), ref[k].view(torch.int32)), k
+
+
+def test_dependent_chain_without_host_sync():
+    # generate -> transpose -> column-wise prefix -> transpose back -> checksum, all queued on one
+    # side stream with no synchronisation: each kernel reads what the previous one wrote
+    n, p = 96, 5000
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        x = bo.generate_prefix(n, p, 41, torch.int32, bo.ROW_WISE, stream=s)
+        xt = bo.transpose(x, stream=s)                                  # [n][p]
+        bo.prefix_sums(xt, bo.COLUMN_WISE, out=xt, stream=s)           # in place
+        y = bo.transpose(xt, stream=s)                                  # [p][n]
+        z = bo.prefix_sums(y, bo.ROW_WISE, stream=s)                    # prefix of the prefix
+    s.synchronize()
+    h = bulkgen.prefix_input(n, p, seed=41, dtype="int32")
+    once = oracle.bulk_prefix_sums(h, oracle.ROW_WISE)
+    twice = oracle.bulk_prefix_sums(once, oracle.ROW_WISE)
+    assert np.array_equal(y.cpu().numpy(), once)
+    assert np.array_equal(z.cpu().numpy(), twice)
