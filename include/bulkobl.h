@@ -87,14 +87,14 @@ typedef enum {
                                instances per warp)                                 */
     BO_TRI_TILED_GLOBAL = 21, /* CTA per instance, same blocked algorithm, table in a
                                per-CTA global workspace slot kept L2-resident
-                               (large n, e.g. 512-gons); workspace
+                               (AUTO for 64 < n < 512); workspace
                                min(p, #SMs) * 16 * (2T^2 + 3T) bytes, T = ceil(n/4) */
     BO_TRI_TILED_QUARTER = 22, /* as BO_TRI_TILED with 8 lanes per instance (four
                                instances per warp; a lane takes several tiles of a
                                tile-diagonal in turn)                             */
     BO_TRI_TILED_GLOBAL8 = 23 /* CTA per instance, 8x8 register tiles over 8-wide
                                table rows read by 256-bit loads, table in a per-CTA
-                               global workspace slot (large n, AUTO for n > 64);
+                               global workspace slot (AUTO for n >= 512);
                                workspace min(p, #SMs) * 32 * (4T^2 + 4T) bytes,
                                T = ceil(n/8), 32-byte aligned                     */
 } bo_variant;
