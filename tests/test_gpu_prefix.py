@@ -165,3 +165,15 @@ def test_column_wise_tma_ring_ragged(dt, n, p):
     x = bulkgen.prefix_input(n, p, seed=n + p, dtype=dt, layout=bulkgen.COLUMN_WISE)
     got = bo.prefix_sums(torch.from_numpy(x).to(DEV), bo.COLUMN_WISE).cpu().numpy()
     assert np.array_equal(got.view(np.uint32), oracle.bulk_prefix_sums(x, oracle.COLUMN_WISE).view(np.uint32))
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+def test_every_small_n_auto(dt, layout):
+    # every n = 1..200 through AUTO (fused-row TMA / smem, across vec4 / scalar), ragged p
+    for n in range(1, 201):
+        p = 61 + (n % 7) * 13
+        x = bulkgen.prefix_input(n, p, seed=2000 + n, dtype=dt, layout=layout)
+        ref = oracle.bulk_prefix_sums(x, layout)
+        got = bo.prefix_sums(torch.from_numpy(x).to(DEV), layout).cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), n

@@ -194,3 +194,16 @@ def test_tr2_large_p_64bit_indexing():
     ids = np.array([0, 2 ** 19 + 3, 2 ** 20 + 7, p - 1])
     ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, seed, "float32"), oracle.ROW_WISE, nthreads=NTHREADS)
     assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+def test_every_n_auto(dt, layout):
+    # every polygon size 3..130 through AUTO (THREAD_REG, TILED_QUARTER, TILED_HALF, TILED_GLOBAL
+    # and their ragged tails), p not a multiple of any tile width
+    for n in range(3, 131):
+        p = 37 + (n % 5)
+        c = bulkgen.tri_input(n, p, seed=1000 + n, dtype=dt, layout=layout)
+        ref = oracle.bulk_opt(c, layout, nthreads=NTHREADS)
+        got = bo.triangulation(torch.from_numpy(c).to(DEV), layout).cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), n
