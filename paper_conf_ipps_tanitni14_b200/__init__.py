@@ -98,7 +98,15 @@ def _dtype_code(t: torch.Tensor) -> int:
     raise TypeError(f"bulkobl supports int32 and float32, got {t.dtype}")
 
 
-def _stream(stream=None) -> int:
+_raw_stream = getattr(torch._C, "_cuda_getCurrentRawStream", None)
+
+
+def _stream(stream=None, t: torch.Tensor | None = None) -> int:
+    """cudaStream_t to launch on: `stream`, else the current stream of t's device
+    (the raw-handle query: torch.cuda.current_stream() builds a Python object
+    and costs ~5 us per call, half of a small call's host time)."""
+    if stream is None and _raw_stream is not None and t is not None and t.is_cuda:
+        return _raw_stream(t.device.index)
     s = stream if stream is not None else torch.cuda.current_stream()
     return s.cuda_stream
 
@@ -139,7 +147,7 @@ def prefix_sums(x: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, ou
             workspace = torch.empty(need, dtype=torch.uint8, device=x.device)
         wptr, wbytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
     _check(lib().bulk_prefix_sums(x.data_ptr(), out.data_ptr(), n, p, dt, layout, variant, wptr, wbytes,
-                                  _stream(stream)))
+                                  _stream(stream, x)))
     return out
 
 
@@ -218,7 +226,7 @@ def triangulation(c: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, 
             workspace = torch.empty(need, dtype=torch.uint8, device=c.device)
         wptr, wbytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
     _check(lib().bulk_triangulation(c.data_ptr(), out.data_ptr(), n, p, dt, layout, variant, wptr, wbytes,
-                                    _stream(stream)))
+                                    _stream(stream, c)))
     return out
 
 
@@ -237,7 +245,7 @@ def triangulation_chords(c: torch.Tensor, layout: int = ROW_WISE, stream=None, o
     if out.dtype != c.dtype or out.numel() != p or chords.dtype != torch.int16 or chords.numel() != p * max(n - 3, 0) * 2:
         raise ValueError("out must be [p] of the weights' dtype and chords [p, n-3, 2] int16")
     _check(lib().bulk_triangulation_chords(c.data_ptr(), out.data_ptr(), chords.data_ptr() if chords.numel() else None,
-                                           n, p, dt, layout, _stream(stream)))
+                                           n, p, dt, layout, _stream(stream, c)))
     return out, chords
 
 
@@ -258,7 +266,7 @@ def execute(program, mem: torch.Tensor, layout: int = COLUMN_WISE, prog_buf: tor
     if prog_buf is None:
         prog_buf = torch.empty(max(t, 1) * 16, dtype=torch.uint8, device=mem.device)
     _check(lib().bulk_execute(code.ctypes.data, t, prog_buf.data_ptr(), prog_buf.numel(), mem.data_ptr(), msize, p,
-                              _dtype_code(mem), layout, nregs, _stream(stream)))
+                              _dtype_code(mem), layout, nregs, _stream(stream, mem)))
     return mem   # pageable H2D copies return once the host program is staged
 
 
@@ -286,7 +294,7 @@ def transpose(x: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> 
     rows, cols = x.shape
     if out is None:
         out = torch.empty((cols, rows), dtype=x.dtype, device=x.device)
-    _check(lib().bulk_transpose(x.data_ptr(), out.data_ptr(), rows, cols, 4, _stream(stream)))
+    _check(lib().bulk_transpose(x.data_ptr(), out.data_ptr(), rows, cols, 4, _stream(stream, x)))
     return out
 
 
@@ -297,7 +305,7 @@ def generate_prefix(n: int, p: int, seed: int, dtype=torch.float32, layout: int 
     if out is None:
         out = torch.empty(shape, dtype=dtype, device=device)
     _check(lib().bulk_generate_prefix(out.data_ptr(), n, p, h0, seed, _dtype_code(out), layout, KINDS[kind],
-                                      _stream(stream)))
+                                      _stream(stream, out)))
     return out
 
 
@@ -307,7 +315,7 @@ def generate_tri(n: int, p: int, seed: int, dtype=torch.float32, layout: int = R
     shape = {ROW_WISE: (p, n, n), COLUMN_WISE: (n, n, p), PACKED_ROW: (p, K), PACKED_COLUMN: (K, p)}[layout]
     if out is None:
         out = torch.empty(shape, dtype=dtype, device=device)
-    _check(lib().bulk_generate_tri(out.data_ptr(), n, p, h0, seed, _dtype_code(out), layout, _stream(stream)))
+    _check(lib().bulk_generate_tri(out.data_ptr(), n, p, h0, seed, _dtype_code(out), layout, _stream(stream, out)))
     return out
 
 
@@ -320,7 +328,7 @@ def checksum(values: torch.Tensor, layout: int = ROW_WISE, h0: int = 0, stream=N
     else:
         n, p = _shape_np(values, layout)
     acc = torch.zeros(1, dtype=torch.int64, device=values.device)
-    _check(lib().bulk_checksum(values.data_ptr(), n, p, h0, layout, acc.data_ptr(), _stream(stream)))
+    _check(lib().bulk_checksum(values.data_ptr(), n, p, h0, layout, acc.data_ptr(), _stream(stream, values)))
     return acc
 
 

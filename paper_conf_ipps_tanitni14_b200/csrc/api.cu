@@ -26,6 +26,31 @@ int cuda_check(cudaError_t e, const char *what) {
     return fail(BO_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
 
+int max_blocks_per_sm(const void *func, int threads, size_t smem) {
+    struct Entry {
+        const void *f;
+        int threads, dev, blocks;
+        size_t smem;
+    };
+    static std::mutex mu;
+    static std::vector<Entry> memo;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        for (const Entry &e : memo)
+            if (e.f == func && e.threads == threads && e.smem == smem && e.dev == dev) return e.blocks;
+    }
+    int blocks = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, func, threads, smem) != cudaSuccess) {
+        cudaGetLastError();
+        blocks = 1;
+    }
+    std::lock_guard<std::mutex> lk(mu);
+    memo.push_back(Entry{func, threads, dev, blocks, smem});
+    return blocks;
+}
+
 bool ensure_dyn_smem(const void *func, int bytes) {
     static std::mutex mu;
     static std::set<std::pair<int, std::pair<const void *, int>>> done;
@@ -54,6 +79,26 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 
 bool make_tmap_2d(CUtensorMap *map, const void *base, uint64_t rows, uint64_t cols, uint32_t box_rows,
                   uint32_t box_cols, CUtensorMapSwizzle swz) {
+    // The encoded map depends only on these arguments, so a repeated call on the
+    // same buffer and shape reuses it: encoding costs several microseconds of
+    // host time, more than a small config's kernel (thread-local, 16 entries).
+    struct Entry {
+        const void *base;
+        uint64_t rows, cols;
+        uint32_t box_rows, box_cols;
+        int swz;
+        CUtensorMap map;
+    };
+    static thread_local Entry memo[16];
+    static thread_local int filled = 0, next = 0;
+    for (int i = 0; i < filled; ++i) {
+        const Entry &e = memo[i];
+        if (e.base == base && e.rows == rows && e.cols == cols && e.box_rows == box_rows && e.box_cols == box_cols &&
+            e.swz == static_cast<int>(swz)) {
+            *map = e.map;
+            return true;
+        }
+    }
     auto fn = encode_fn();
     if (!fn) return false;
     cuuint64_t dims[2] = {cols, rows};
@@ -63,7 +108,11 @@ bool make_tmap_2d(CUtensorMap *map, const void *base, uint64_t rows, uint64_t co
     CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void *>(base), dims, strides, box, es,
                     CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    return r == CUDA_SUCCESS;
+    if (r != CUDA_SUCCESS) return false;
+    memo[next] = Entry{base, rows, cols, box_rows, box_cols, static_cast<int>(swz), *map};
+    next = (next + 1) % 16;
+    filled = filled < 16 ? filled + 1 : 16;
+    return true;
 }
 
 // ---------------------------------------------------------------- internals

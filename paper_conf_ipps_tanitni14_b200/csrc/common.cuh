@@ -61,6 +61,11 @@ inline void launch(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem,
 // done once per (device, kernel) -- processes may drive several GPUs.
 bool ensure_dyn_smem(const void *func, int bytes);
 
+// Resident CTAs per SM of `func` at this block size and dynamic shared memory,
+// memoised per (device, kernel, threads, smem): the occupancy query is a
+// per-call host cost the small configs (a few microseconds of GPU time) feel.
+int max_blocks_per_sm(const void *func, int threads, size_t smem);
+
 inline int num_sms() {
     static int sms = [] {
         int dev = 0, v = 148;

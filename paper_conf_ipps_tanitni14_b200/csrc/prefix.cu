@@ -429,7 +429,7 @@ static int launch_across_tma(const T *src, T *dst, int64_t n, int64_t p, cudaStr
     const long long ntiles = (p + INST - 1) / INST;
     const int nchunks = static_cast<int>((n + ac::kElems - 1) / ac::kElems);
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ps_across_tma<T, INST>, INST, C::kSmem);
+    per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&ps_across_tma<T, INST>), INST, C::kSmem);
     const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
     const int slot = fr_next_slot();
     launch(ps_across_tma<T, INST>, static_cast<unsigned>(grid), INST, C::kSmem, st, smap, dmap, ntiles, nchunks, slot);
@@ -476,7 +476,7 @@ static int launch_fused_row_tma(const T *src, T *dst, int64_t n, int64_t p, cuda
     const long long ntiles = (p + INST - 1) / INST;
     const int nchunks = static_cast<int>((n + fr::kElems - 1) / fr::kElems);
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, ps_fused_row_tma<T, INST>, INST, C::kSmem);
+    per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&ps_fused_row_tma<T, INST>), INST, C::kSmem);
     const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
     const int slot = fr_next_slot();
     launch(ps_fused_row_tma<T, INST>, static_cast<unsigned>(grid), INST, C::kSmem, st, smap, dmap, ntiles, nchunks,

@@ -156,7 +156,7 @@ int launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, cud
         const long long tiles_r = (rows + tr::kRows - 1) / tr::kRows;
         const long long ntiles = tiles_c * tiles_r;
         int per_sm = 1;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, transpose_tma_kernel, tr::kThreads, tr::kSmem);
+        per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&transpose_tma_kernel), tr::kThreads, tr::kSmem);
         const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
         static std::atomic<unsigned> next_slot{0};
         const int slot = static_cast<int>(next_slot.fetch_add(1) % kWorkSlots);

@@ -384,7 +384,7 @@ static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) 
     if (!attr) return fail(BO_ECUDA, "triangulation THREAD_REG: cannot set dynamic smem");
     const long long nbatch = (p + 31) / 32;
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * W, smem);
+    per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(kern), 32 * W, smem);
     // enough CTAs that every warp of every resident CTA has a batch
     const long long grid = std::min<long long>((nbatch + W - 1) / W, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
     launch(kern, static_cast<unsigned>(grid), 32 * W, smem, st, map, static_cast<T *>(out), p, nbatch);
@@ -400,7 +400,7 @@ static int launch_reg_packed(const void *c, void *out, int64_t p, cudaStream_t s
     if (!attr) return fail(BO_ECUDA, "triangulation THREAD_REG packed: cannot set dynamic smem");
     const long long nbatch = (p + 31) / 32;
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_thread_reg_packed<T, N>, 32, smem);
+    per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&tri_thread_reg_packed<T, N>), 32, smem);
     const long long grid = std::min<long long>(nbatch, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
     launch(tri_thread_reg_packed<T, N>, static_cast<unsigned>(grid), 32, smem, st, 
         static_cast<const T *>(c), static_cast<T *>(out), p, nbatch);
@@ -451,7 +451,7 @@ static int launch_smem_warp(const void *c, void *out, int64_t n, int64_t p, int 
     W = std::max(W, 1);
     const size_t smem = W * per;
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_smem_warp<T>, W * 32, smem);
+    per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&tri_smem_warp<T>), W * 32, smem);
     per_sm = std::max(per_sm, 1);
     const long long blocks = std::min<long long>((p + W - 1) / W, static_cast<long long>(per_sm) * num_sms() * 8);
     launch(tri_smem_warp<T>, static_cast<unsigned>(blocks), W * 32, smem, st, 

@@ -689,7 +689,7 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
     const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_tiled_kernel<T, LPI, CHORDS>), 227 * 1024);
     if (!attr) return fail(BO_ECUDA, "tiled: cannot set dynamic smem");
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tri_tiled_kernel<T, LPI, CHORDS>, W * 32, smem);
+    per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&tri_tiled_kernel<T, LPI, CHORDS>), W * 32, smem);
     per_sm = std::max(per_sm, 1);
     const long long per_cta = static_cast<long long>(W) * IPW;
     const long long blocks = std::min<long long>((p + per_cta - 1) / per_cta,
