@@ -367,7 +367,8 @@ def tri_roofline(wl, per_launch_ms, peaks):
     tops = addmin_per_instance(wl) * p / secs / 1e12
     alu = alu_peak_taddmin(peaks, wl["dtype"])
     hbm = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": gbs / peaks["hbm_gbs"]}
-    alu_r = {"bound": "alu", "achieved": tops, "peak": alu, "unit": "T add-min/s", "frac": tops / alu}
+    alu_r = {"bound": "alu", "achieved": tops, "peak": alu, "unit": "T add-min/s", "frac": tops / alu,
+             "peak_source": "measured inner mix, tools/micro/addmin_peak.cu (profiles/r01/addmin_peak.log)"}
     t_hbm = algo_bytes_per_instance(wl) * p / (peaks["hbm_gbs"] * 1e9)
     t_alu = addmin_per_instance(wl) * p / (alu * 1e12)
     main, other = (hbm, alu_r) if t_hbm >= t_alu else (alu_r, hbm)
@@ -378,12 +379,16 @@ def tri_roofline(wl, per_launch_ms, peaks):
 
 
 def alu_peak_taddmin(peaks, dtype):
-    """ALU roof for the min-plus inner step: 148 SMs x 4
-    SMSPs x 32 lanes x f_max, one add-min per lane per cycle (fp32: FADD2 +
-    FMNMX3 = 2 issue slots per 2 add-mins; int32: one VIADDMNMX, same issue
-    rate assumed)."""
+    """ALU roof for the min-plus inner step, MEASURED (SURVEY §8 d: R_addmin from a
+    microbenchmark of the actual inner instruction mix): tools/micro/addmin_peak.cu
+    runs the 4x4 chunk of tri_tiled.cu from registers on all 148 SMs --
+    fp32 FADD2 + FMNMX3 68.5, int32 VIADDMNMX 61.5 add-mins per SM per clock
+    (profiles/r01/addmin_peak.log); scaled by the SM count and max clock.
+    (One add-min per lane per cycle, 128 per SM-clock, is what the unit counts
+    suggest; the measured mix reaches half of it.)"""
     mhz = peaks.get("sm_max_mhz", 1965.0)
-    return 148 * 128 * mhz * 1e6 / 1e12
+    per_sm_clk = 68.5 if dtype == "float32" else 61.5
+    return 148 * per_sm_clk * mhz * 1e6 / 1e12
 
 
 def cpu_baseline(ctx, name, st, budget_s=12.0):
