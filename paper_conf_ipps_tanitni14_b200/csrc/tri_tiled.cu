@@ -242,8 +242,8 @@ __device__ __forceinline__ void fixup<float>(float (&t)[4][4], const float (&S)[
 }
 
 // Dense part of tile (I, J) over chunk-columns m, m + s, ... < J (m < J):
-// software-pipelined ping-pong (load chunk m+s while computing chunk m); the
-// first chunk initialises acc (no +inf fill).
+// software-pipelined ping-pong (load chunk m+s while computing chunk m); acc
+// arrives filled with +inf.
 template <typename T>
 __device__ __forceinline__ void dense_tile(T (&acc)[4][4], const T *Z, int I, int J, int m, int s) {
     using T4 = typename V4<T>::type;
@@ -261,7 +261,7 @@ __device__ __forceinline__ void dense_tile(T (&acc)[4][4], const T *Z, int I, in
 #pragma unroll
         for (int u = 0; u < 4; ++u) A1[u] = ld4(pa + 4 * u), B1[u] = ld4(pb + 4 * u);
     }
-    minplus_first(acc, A0, B0);
+    minplus_chunk(acc, A0, B0);
     while (more) {
         pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
         pb += db;
@@ -572,14 +572,13 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             const bool act = I < NT - D;
             const int J = I + D;
             T acc[4][4];
-            if (act && I + 1 + q < J) {
-                tt::dense_tile(acc, Z, I, J, I + 1 + q, s);
-            } else {
+            // every lane starts from +inf (uniform, no divergent init branch: -1 %
+            // against initialising from the first chunk)
 #pragma unroll
-                for (int u = 0; u < 4; ++u)
+            for (int u = 0; u < 4; ++u)
 #pragma unroll
-                    for (int v = 0; v < 4; ++v) acc[u][v] = Op::inf();
-            }
+                for (int v = 0; v < 4; ++v) acc[u][v] = Op::inf();
+            if (act && I + 1 + q < J) tt::dense_tile(acc, Z, I, J, I + 1 + q, s);
             BO_CLK_MARK(80 + 4 * D);
             for (int off = 1 << ib; off < LPI; off <<= 1)
 #pragma unroll
