@@ -59,6 +59,8 @@ WORKLOADS = {
                 desc="bulk optimal triangulation int32 n=16, p=65536 (BASELINE configs[2])"),
     "tr2": dict(seed=4, algo="tri", n=64, p=65536, dtype="float32", layout=0, variant=0,
                 desc="bulk optimal triangulation fp32 n=64, p=65536 (BASELINE configs[3])"),
+    "tr2col": dict(seed=4, algo="tri", n=64, p=65536, dtype="float32", layout=1, variant=0,
+                   desc="TR-2 with the weights in the paper's column-wise arrangement [n][n][p] (P:212)"),
     "tr2umm": dict(seed=4, algo="tri", n=64, p=65536, dtype="float32", layout=1, variant=16,
                    desc="the paper's column-wise UMM kernel on TR-2"),
     "tr1col": dict(seed=3, algo="tri", n=16, p=65536, dtype="int32", layout=1, variant=0,
@@ -80,7 +82,7 @@ WORKLOADS = {
     "ps2naive_row": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=5,
                          desc="the paper's row-wise kernel (thread per instance, uncoalesced)"),
 }
-EXTRAS = ["ps2col", "ps2tr", "tr_transpose", "ps1", "tr1", "tr1col", "tr1packed", "tr2", "tr2packed", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
+EXTRAS = ["ps2col", "ps2tr", "tr_transpose", "ps1", "tr1", "tr1col", "tr1packed", "tr2", "tr2col", "tr2packed", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
           "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col"]
 L2_BYTES = 126 * 2 ** 20
 
