@@ -2,7 +2,14 @@
 """bench.py -- bulk execution of oblivious algorithms on B200 (libbulkobl).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--workload ps2|ps2col|ps1|tr1|tr2]
-                    [--impl ours|reference] [--no-extras] [--no-cpu-baseline]
+                    [--impl ours|reference] [--no-extras] [--no-cpu-baseline] [--sweep]
+                    [--dist-backend nccl|gloo]
+
+--gpus N > 1 without WORLD_SIZE in the environment re-executes this script
+under `torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1`
+(one rank per GPU); under torchrun the world size must equal N.  --sweep runs
+BASELINE configs[4] (p = 2^10..2^22 per rank, both algorithms) instead of the
+headline workload.
 
 Headline workload (BASELINE.json configs[1]): bulk prefix sums, fp32, n=1024,
 p=2^20 instances PER GPU (weak scaling; rank r owns global instances
@@ -190,6 +197,33 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
+def _free_port():
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    return port
+
+
+def self_launch_argv(gpus, argv, port):
+    """The torchrun command line `--gpus N` (N > 1, no WORLD_SIZE set) re-executes
+    bench.py under: one rank per GPU, rendezvous on 127.0.0.1."""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={gpus}",
+            "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *argv]
+
+
+def maybe_self_launch(args, argv):
+    """Returns None when this process is a rank to run; else the exit code of the
+    torchrun child this process spawned for `--gpus N`."""
+    if args.gpus is None or args.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return None
+    if args.impl == "reference":          # the CPU arm: rank 0 alone does work
+        return None
+    import subprocess
+    return subprocess.call(self_launch_argv(args.gpus, argv, _free_port()))
+
+
 class Ctx:
     def __init__(self, backend="nccl"):
         self.rank = int(os.environ.get("RANK", 0))
@@ -308,8 +342,11 @@ def setup_workload(wl, rank, copies=1):
 
         nxt = _rotator(x, copies)
 
+        def fn_on(src):
+            bo.prefix_sums(src, wl["layout"], wl["variant"], out=out, workspace=ws)
+
         def fn():
-            bo.prefix_sums(nxt(), wl["layout"], wl["variant"], out=out, workspace=ws)
+            fn_on(nxt())
         variant = bo.prefix_sums_variant(n, p, bo.F32 if wl["dtype"] == "float32" else bo.I32, wl["layout"],
                                          wl["variant"])
     else:
@@ -324,10 +361,14 @@ def setup_workload(wl, rank, copies=1):
         need = bo.triangulation_workspace(n, p, dcode, wl["layout"], wl["variant"])
         ws = torch.empty(need, dtype=torch.uint8, device="cuda") if need else None
 
+        def fn_on(src):
+            bo.triangulation(src, wl["layout"], wl["variant"], out=out, workspace=ws)
+
         def fn():
-            bo.triangulation(nxt(), wl["layout"], wl["variant"], out=out, workspace=ws)
+            fn_on(nxt())
         variant = bo.triangulation_variant(n, p, dcode, wl["layout"], wl["variant"])
-    return dict(x=x, out=out, fn=fn, seed=seed, h0=h0, variant=bo.VARIANT_NAMES.get(variant, str(variant)))
+    return dict(x=x, out=out, fn=fn, fn_on=fn_on, seed=seed, h0=h0,
+                variant=bo.VARIANT_NAMES.get(variant, str(variant)))
 
 
 def input_bytes(wl):
@@ -533,6 +574,38 @@ def e2e(ctx, name, steps, warmup):
             "gpu_launches": bo.launch_count() - c0}
 
 
+def single_gpu_checksums(wl, st, world):
+    """Per-shard checksums of the whole problem computed on THIS GPU alone: shard r
+    (global ids [r*p, (r+1)*p)) is regenerated into rank 0's input buffer and run
+    with the same call, one shard after the other.  Equal to the all-gathered
+    per-rank checksums iff the multi-rank run computed what one GPU computes."""
+    import paper_conf_ipps_tanitni14_b200 as bo
+    n, p = wl["n"], wl["p"]
+    dt = getattr(torch, wl["dtype"])
+    x, out = st["x"], st["out"]
+    res = []
+    for r in range(world):
+        h0 = r * p
+        if wl["algo"] == "prefix":
+            bo.generate_prefix(n, p, wl["seed"], dt, wl["layout"], "uniform", h0=h0, out=x)
+        elif wl["algo"] == "tri":
+            bo.generate_tri(n, p, wl["seed"], dt, wl["layout"], h0=h0, out=x)
+        else:
+            return []
+        st["fn_on"](x)
+        cs = bo.checksum(out, wl["layout"] if wl["algo"] == "prefix" else 0, h0=h0)
+        res.append(int(cs.cpu().numpy().view(np.uint64)[0]))
+    # leave rank 0's own shard in place again
+    if world > 1:
+        if wl["algo"] == "prefix":
+            bo.generate_prefix(n, p, wl["seed"], dt, wl["layout"], "uniform", h0=st["h0"], out=x)
+        else:
+            bo.generate_tri(n, p, wl["seed"], dt, wl["layout"], h0=st["h0"], out=x)
+        st["fn_on"](x)
+    torch.cuda.synchronize()
+    return res
+
+
 def run_ours(args, ctx):
     import paper_conf_ipps_tanitni14_b200 as bo
     bo.lib()
@@ -582,8 +655,20 @@ def run_ours(args, ctx):
     cs_list = shard.gather_checksums(int(cs.cpu().numpy().view(np.uint64)[0]))
     line["checksums"] = {"per_rank": [hex(c) for c in cs_list],
                          "combined": hex(shard.combine_checksums(cs_list)),
-                         "note": "one NCCL all-gather after the timed region; inputs are generated per rank "
+                         "note": "one all-gather after the timed region; inputs are generated per rank "
                                  "from global instance ids, so nothing crosses NVLink on the data path"}
+    # the oracle on a sample of rank 0's shard (before anything reuses st's buffers)
+    if args.cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(ctx, name, st) if ctx.rank == 0 else None
+    # G-invariance: rank 0 recomputes every rank's shard on its own GPU, one after
+    # the other (what a single-GPU run of the whole problem computes), and compares
+    if ctx.rank == 0 and wl["algo"] in ("prefix", "tri") and "fn_on" in st:
+        single = single_gpu_checksums(wl, st, ctx.world)
+        line["checksums"]["single_gpu_recompute"] = [hex(c) for c in single]
+        line["checksums_match"] = single == cs_list
+        if "cpu_baseline" in line and line["cpu_baseline"]:
+            line["checksums_match_oracle_sample"] = line["cpu_baseline"]["gpu_matches_oracle_on_sample"]
+    ctx.barrier()
     if args.extras:
         ex = {}
         for e in EXTRAS:
@@ -602,11 +687,76 @@ def run_ours(args, ctx):
             line["e2e"] = e2e(ctx, name, max(2, min(args.steps, 5)), 1)
         except Exception as exc:                    # e.g. pinned host memory exhausted at 8 ranks
             line["e2e"] = {"error": repr(exc)}
-    if args.cpu_baseline and ctx.rank == 0 and ctx.world == 1:
-        line["cpu_baseline"] = cpu_baseline(ctx, name, st)
-    elif args.cpu_baseline:
-        line["cpu_baseline"] = None
     if ctx.rank == 0:
+        print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------ p-sweep
+SWEEP_CASES = [("prefix", 32, "int32", 1), ("prefix", 1024, "float32", 2), ("tri", 16, "int32", 3),
+               ("tri", 64, "float32", 4)]
+
+
+def run_sweep(args, ctx):
+    """BASELINE configs[4]: p = 2^lo..2^hi instances PER RANK (weak scaling) for
+    both algorithms at the configs' n and dtype, AUTO variant, row-wise inputs,
+    timed like the headline (max over ranks).  Every point all-gathers the shard
+    checksums, compares them with rank 0's single-GPU recomputation of every
+    shard, and checks sampled instances of rank 0's shard against the oracle."""
+    import bulkgen
+    import oracle
+    import paper_conf_ipps_tanitni14_b200 as bo
+    from paper_conf_ipps_tanitni14_b200 import shard
+    bo.lib()
+    lo, hi, step = (int(v) for v in args.sweep_log2.split(":"))
+    peaks, _ = load_peaks()
+    stream = torch.cuda.Stream()
+    points = []
+    sampler = ClockSampler(ctx.device)
+    with sampler:
+        for algo, n, dt, seed in SWEEP_CASES:
+            for lg in range(lo, hi + 1, step):
+                p = 2 ** lg
+                wl = dict(seed=seed, algo=algo, n=n, p=p, dtype=dt, layout=0, variant=0, desc="sweep")
+                st = setup_workload(wl, ctx.rank, copies_for(wl))
+                ms, launches = timed(ctx, st["fn"], max(5, min(args.steps, 20)), args.warmup, stream)
+                st["fn_on"](st["x"])
+                cs = bo.checksum(st["out"], 0, h0=st["h0"])
+                parts = shard.gather_checksums(int(cs.cpu().numpy().view(np.uint64)[0]))
+                pt = {"algo": algo, "n": n, "dtype": dt, "p_per_gpu": p, "p_total": p * ctx.world,
+                      "variant": st["variant"], "ms_per_step": ms, "value": p * ctx.world / (ms * 1e-3),
+                      "unit": UNIT, "gpu_launches": launches}
+                if algo == "prefix":
+                    gbs = algo_bytes_per_instance(wl) * p / (ms * 1e-3) / 1e9
+                    pt["GBps_per_gpu"] = gbs
+                    pt["hbm_frac"] = gbs / peaks["hbm_gbs"]
+                else:
+                    pt["T_addmin_per_gpu"] = addmin_per_instance(wl) * p / (ms * 1e-3) / 1e12
+                if ctx.rank == 0:
+                    single = single_gpu_checksums(wl, st, ctx.world)
+                    pt["checksums_match"] = single == parts
+                    rng = np.random.default_rng(lg)
+                    loc = np.unique(np.r_[rng.integers(0, p, 6), 0, p - 1])
+                    ids = loc + st["h0"]
+                    if algo == "prefix":
+                        ref = oracle.bulk_prefix_sums(bulkgen.prefix_instances(n, ids, seed, dt), oracle.ROW_WISE)
+                    else:
+                        ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, seed, dt), oracle.ROW_WISE)
+                    got = st["out"][torch.from_numpy(loc).cuda()].cpu().numpy()
+                    pt["oracle_sample_match"] = bool(np.array_equal(np.ascontiguousarray(got).view(np.uint32),
+                                                                    ref.view(np.uint32)))
+                ctx.barrier()
+                points.append(pt)
+                del st
+                torch.cuda.empty_cache()
+    if ctx.rank == 0:
+        line = {"mode": "sweep", "metric": METRIC, "unit": UNIT, "n_gpus": ctx.world, "scaling": "weak",
+                "higher_is_better": True, "data": "synthetic", "steps": max(5, min(args.steps, 20)),
+                "warmup": args.warmup,
+                "config": {"workload": "BASELINE configs[4]: p-sweep per GPU, both algorithms, AUTO variants",
+                           "log2_p": [lo, hi, step]},
+                "all_checksums_match": all(pt.get("checksums_match", True) for pt in points),
+                "all_oracle_samples_match": all(pt.get("oracle_sample_match", True) for pt in points),
+                "clocks": sampler.summary(), "points": points}
         print(json.dumps(line), flush=True)
 
 
@@ -666,9 +816,10 @@ def run_reference(args, ctx):
     print(json.dumps(line), flush=True)
 
 
-def main():
+def main(argv=None):
     ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--gpus", type=int, default=None,
+                    help="ranks (one per GPU); default: WORLD_SIZE under torchrun, else 1")
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--workload", default="ps2", choices=sorted(k for k in WORKLOADS if WORKLOADS[k]["algo"] != "transpose"))
@@ -678,13 +829,26 @@ def main():
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo only to test the multi-rank logic with several ranks on one GPU")
-    args = ap.parse_args()
+    ap.add_argument("--sweep", action="store_true", help="BASELINE configs[4]: p = 2^10..2^22 per rank")
+    ap.add_argument("--sweep-log2", default="10:22:2", help="lo:hi:step of log2(p) for --sweep")
+    args = ap.parse_args(argv)
     if args.warmup < 3:
         args.warmup = 3
+    rc = maybe_self_launch(args, sys.argv[1:] if argv is None else argv)
+    if rc is not None:
+        sys.exit(rc)
     ctx = Ctx(args.dist_backend)
     if args.impl == "reference":
+        if args.gpus and not ctx.dist:
+            ctx.world = args.gpus                # reported; the CPU arm's work does not depend on it
         run_reference(args, ctx)
         return
+    if args.gpus is not None and args.gpus != ctx.world:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ctx.world}")
+    if ctx.dist and ctx.backend == "nccl" and torch.cuda.device_count() < ctx.world:
+        raise SystemExit(f"bench.py: {ctx.world} NCCL ranks need {ctx.world} GPUs, this node has "
+                         f"{torch.cuda.device_count()} (use --dist-backend gloo to test the multi-rank "
+                         "logic with several ranks per GPU)")
     torch.cuda.set_device(ctx.device)
     if ctx.dist:
         if ctx.backend == "nccl":
@@ -692,7 +856,10 @@ def main():
         else:
             dist.init_process_group(ctx.backend)
     try:
-        run_ours(args, ctx)
+        if args.sweep:
+            run_sweep(args, ctx)
+        else:
+            run_ours(args, ctx)
     finally:
         if ctx.dist:
             ctx.barrier()

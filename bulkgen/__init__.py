@@ -19,11 +19,21 @@ Prefix-sum inputs (paper: "float (32-bit) numbers", Sec. V):
     'ones':           1                         (closed-form pin 1..n)
     'arange':         e                         (closed-form pin e(e+1)/2)
     'smallint':       (u >> 60)                 integers 0..15 (exact in fp32)
-Triangulation chord weights (dense n x n per instance, reading G6):
+Triangulation chord weights (dense n x n per instance, reading G6),
+e = a*n + b, two kinds:
+  'chords' (the configs' workload; TR_KINDS code 0):
     c[a][b] for b-a >= 2 and (a,b) != (0,n-1):
         int32: u >> 44  in [0, 2^20)            fp32: (u >> 40) * 2^-24
     every other entry (polygon sides, root side, lower triangle) = 0 (G8)
-    with e = a*n + b.
+  'full' (parity stress; code 1): EVERY entry is non-zero.
+    read entries b-a >= 2, INCLUDING the root side c[0][n-1] (P:199 adds it):
+        int32: (u >> 32) mod (2B-1) - (B-1), B = 2^31 div (2(n-2)), signed,
+               so |c| < 2^31 / (2(n-2)) (the ABI bound, reading G13)
+        fp32:  (u >> 40) * 2^-23 - 1            signed, in [-1, 1)
+    unread entries b-a <= 1 (sides, diagonal, lower triangle) hold poison:
+        int32: (int32)(u >> 32) (full range)
+        fp32:  by u >> 61: qNaN, +inf, -inf, +FLT_MAX, -FLT_MAX, sNaN, -0,
+               a value in [-1, 1) -- any read of them changes the result
 """
 from __future__ import annotations
 
@@ -96,22 +106,46 @@ def prefix_instances(n: int, ids, seed: int, dtype: str = "float32", kind: str =
     return np.ascontiguousarray(_prefix_values(u64(seed, h, e), e, dtype, kind))
 
 
-def _tri_values(n: int, u: np.ndarray, dtype: str) -> np.ndarray:
+TR_KINDS = {"chords": 0, "full": 1}
+# fp32 poison for the entries Algorithm OPT never reads ('full' kind), by u >> 61
+_F32_POISON = np.array([0x7FC00000, 0x7F800000, 0xFF800000, 0x7F7FFFFF, 0xFF7FFFFF, 0x7FA00000, 0x80000000, 0],
+                       dtype=np.uint32)
+
+
+def tri_int32_bound(n: int) -> int:
+    """B = 2^31 div (2(n-2)): 'full' int32 weights satisfy |c| <= B-1 (reading G13)."""
+    return (1 << 31) // (2 * max(n - 2, 1))
+
+
+def _tri_values(n: int, u: np.ndarray, dtype: str, kind: str = "chords") -> np.ndarray:
     a = np.arange(n)[:, None]
     b = np.arange(n)[None, :]
-    mask = (b - a >= 2) & ~((a == 0) & (b == n - 1))
+    if kind == "chords":
+        mask = (b - a >= 2) & ~((a == 0) & (b == n - 1))
+        if dtype == "int32":
+            v = (u >> np.uint64(44)).astype(np.int32)
+        else:
+            v = ((u >> np.uint64(40)).astype(np.float64) * 2.0 ** -24).astype(np.float32)
+        return np.where(mask, v, np.zeros((), dtype=v.dtype))
+    if kind != "full":
+        raise ValueError(f"unknown kind {kind!r}")
+    read = np.broadcast_to(b - a >= 2, u.shape)
     if dtype == "int32":
-        v = (u >> np.uint64(44)).astype(np.int32)
-    else:
-        v = ((u >> np.uint64(40)).astype(np.float64) * 2.0 ** -24).astype(np.float32)
-    return np.where(mask, v, np.zeros((), dtype=v.dtype))
+        B = tri_int32_bound(n)
+        v = ((u >> np.uint64(32)) % np.uint64(2 * B - 1)).astype(np.int64) - (B - 1)
+        poison = (u >> np.uint64(32)).astype(np.uint32).view(np.int32)
+        return np.where(read, v.astype(np.int32), poison)
+    v = ((u >> np.uint64(40)).astype(np.float64) * 2.0 ** -23 - 1.0).astype(np.float32)
+    pb = _F32_POISON[(u >> np.uint64(61)).astype(np.int64)]
+    pb = np.where(pb == 0, v.view(np.uint32), pb)
+    return np.where(read, v, pb.view(np.float32))
 
 
-def tri_instances(n: int, ids, seed: int, dtype: str = "float32") -> np.ndarray:
+def tri_instances(n: int, ids, seed: int, dtype: str = "float32", kind: str = "chords") -> np.ndarray:
     """Chord weights of selected instances, shape [len(ids), n, n]."""
     h = np.asarray(ids, dtype=np.uint64)[:, None, None]
     e = np.arange(n * n, dtype=np.uint64).reshape(1, n, n)
-    return np.ascontiguousarray(_tri_values(n, u64(seed, h, e), dtype))
+    return np.ascontiguousarray(_tri_values(n, u64(seed, h, e), dtype, kind))
 
 
 def packed_pairs(n: int):
@@ -121,10 +155,10 @@ def packed_pairs(n: int):
 
 
 def tri_input(n: int, p: int, seed: int, dtype: str = "float32", layout: int = ROW_WISE,
-              h0: int = 0) -> np.ndarray:
+              h0: int = 0, kind: str = "chords") -> np.ndarray:
     """Chord weights: ROW_WISE [p, n, n] (c[h*n*n + a*n + b]), COLUMN_WISE
     [n, n, p] (c[(a*n + b)*p + h]), PACKED_ROW [p, K], PACKED_COLUMN [K, p]."""
-    v = tri_instances(n, np.arange(h0, h0 + p), seed, dtype)
+    v = tri_instances(n, np.arange(h0, h0 + p), seed, dtype, kind)
     if layout == ROW_WISE:
         return v
     if layout == COLUMN_WISE:

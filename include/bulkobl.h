@@ -121,15 +121,18 @@ size_t bulk_prefix_sums_workspace(int64_t n, int64_t p, int dtype, int layout, i
 /* That is the minimum total chord weight over all triangulations */
 /* PLUS c[0, n-1] (the root side v0 v_{n-1}, which Algorithm OPT adds; set it */
 /* to 0 to get the pure chord total).  Only entries c[a][b] with b-a >= 2 are */
-/* read.                                                                       */
+/* read: the polygon sides c[a][a+1], the diagonal and the lower triangle    */
+/* may hold anything (NaN, inf, garbage) -- they never reach the result.      */
 /*   c   : device, dense n x n weights per instance.  Row-wise:               */
 /*         c[h*n*n + a*n + b];  column-wise: c[(a*n + b)*p + h], */
 /*         or packed (BO_PACKED_ROW / BO_PACKED_COLUMN, see bo_layout).       */
 /*   out : device, p elements of dtype.                                       */
 /*   n >= 3 (n < 3 is BO_EINVAL), p >= 0; n <= 4096.                          */
-/*   int32 weights must satisfy |c| < 2^31 / (2(n-2)) (no overflow); fp32     */
-/*   weights must be finite and >= 0 (results are then bit-identical to the   */
-/*   sequential algorithm: min is exact, every sum keeps its association).    */
+/*   The entries read (b-a >= 2) may be negative.  int32 weights must satisfy */
+/*   |c| < 2^31 / (2(n-2)) (no overflow); fp32 weights must be finite with    */
+/*   |c| < FLT_MAX / (2(n-2)) (no sum overflows).  Results are then           */
+/*   bit-identical to the sequential algorithm: min is exact, every sum keeps */
+/*   its association, and no table value is ever -0 (reading G16). */
 /*   workspace: device, >= bulk_triangulation_workspace(...) bytes (only      */
 /*   BO_TRI_UMM_GLOBAL needs one).                                            */
 /* ------------------------------------------------------------------------- */
@@ -204,12 +207,16 @@ int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, 
 /* Synthetic inputs, generated on the device by the counter-based generator  */
 /* documented in bulkgen/__init__.py (same bits on host and device):         */
 /*   u = mix64(seed*K_SEED + h*K_H + e*K_E), h = GLOBAL instance id h0+local. */
-/* kind: 0 uniform, 1 ones, 2 arange, 3 smallint (prefix only).               */
+/* prefix kind: 0 uniform, 1 ones, 2 arange, 3 smallint.                    */
+/* triangulation kind: 0 'chords' (non-negative chord weights; polygon sides, */
+/*   root side and lower triangle 0 -- the configs' workload), 1 'full'        */
+/*   (signed weights on every entry read, root side included; poison --       */
+/*   NaN, +-inf, +-FLT_MAX, -0, garbage int32 -- on every entry never read).  */
 /* ------------------------------------------------------------------------- */
 int bulk_generate_prefix(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype,
                          int layout, int kind, void *stream);
 int bulk_generate_tri(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype,
-                      int layout, void *stream);
+                      int layout, int kind, void *stream);
 
 /* Order-independent checksum of a result (values: [p][n] row-wise, [n][p]   */
 /* column-wise; n = 1 for per-instance results):                             */

@@ -36,6 +36,7 @@ VARIANT_NAMES = {
     TRI_TILED_GLOBAL8: "tiled_global8",
 }
 KINDS = {"uniform": 0, "ones": 1, "arange": 2, "smallint": 3}
+TR_KINDS = {"chords": 0, "full": 1}
 
 
 class BulkError(RuntimeError):
@@ -69,7 +70,7 @@ def lib() -> ctypes.CDLL:
             "bulk_prefix_sums_host_bytes": ([i64, i64, i32, i32, i32], sz),
             "bulk_triangulation_host_bytes": ([i64, i64, i32, i32, i32], sz),
             "bulk_generate_prefix": ([vp, i64, i64, i64, u64, i32, i32, i32, vp], i32),
-            "bulk_generate_tri": ([vp, i64, i64, i64, u64, i32, i32, vp], i32),
+            "bulk_generate_tri": ([vp, i64, i64, i64, u64, i32, i32, i32, vp], i32),
             "bulk_checksum": ([vp, i64, i64, i64, i32, vp, vp], i32),
             "bulk_last_error": ([], ctypes.c_char_p),
             "bulk_prefix_sums_variant": ([i64, i64, i32, i32, i32, vp, vp], i32),
@@ -310,12 +311,13 @@ def generate_prefix(n: int, p: int, seed: int, dtype=torch.float32, layout: int 
 
 
 def generate_tri(n: int, p: int, seed: int, dtype=torch.float32, layout: int = ROW_WISE, h0: int = 0,
-                 device="cuda", out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+                 device="cuda", out: torch.Tensor | None = None, stream=None, kind: str = "chords") -> torch.Tensor:
     K = (n - 1) * (n - 2) // 2
     shape = {ROW_WISE: (p, n, n), COLUMN_WISE: (n, n, p), PACKED_ROW: (p, K), PACKED_COLUMN: (K, p)}[layout]
     if out is None:
         out = torch.empty(shape, dtype=dtype, device=device)
-    _check(lib().bulk_generate_tri(out.data_ptr(), n, p, h0, seed, _dtype_code(out), layout, _stream(stream, out)))
+    _check(lib().bulk_generate_tri(out.data_ptr(), n, p, h0, seed, _dtype_code(out), layout, TR_KINDS[kind],
+                                   _stream(stream, out)))
     return out
 
 

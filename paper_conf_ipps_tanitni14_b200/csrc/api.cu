@@ -128,7 +128,7 @@ int launch_tri_chords(const void *c, void *out, int16_t *chords, int64_t n, int6
                       cudaStream_t st);
 size_t tri_workspace(int64_t n, int64_t p, int variant);
 int launch_gen_prefix(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
-int launch_gen_tri(void *, int64_t, int64_t, int64_t, uint64_t, int, int, cudaStream_t);
+int launch_gen_tri(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
 int launch_checksum(const void *, int64_t, int64_t, int64_t, int, uint64_t *, cudaStream_t);
 int launch_exec(const void *prog, int64_t t, void *mem, int64_t msize, int64_t p, int dtype, int layout, int nregs,
                 cudaStream_t st);
@@ -349,13 +349,13 @@ int bulk_generate_prefix(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t s
 }
 
 int bulk_generate_tri(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout,
-                      void *stream) {
+                      int kind, void *stream) {
     t_err.clear();
-    if (n < 1 || p < 0 || h0 < 0 || !valid_dtype(dtype) || !valid_tri_layout(layout) ||
+    if (n < 1 || p < 0 || h0 < 0 || !valid_dtype(dtype) || !valid_tri_layout(layout) || kind < 0 || kind > 1 ||
         (layout >= BO_PACKED_ROW && n < 3))
         return fail(BO_EINVAL, "generate_tri: bad argument");
     if (p > 0 && !dst) return fail(BO_EINVAL, "generate_tri: NULL pointer");
-    return launch_gen_tri(dst, n, p, h0, seed, dtype, layout, static_cast<cudaStream_t>(stream));
+    return launch_gen_tri(dst, n, p, h0, seed, dtype, layout, kind, static_cast<cudaStream_t>(stream));
 }
 
 int bulk_checksum(const void *values, int64_t n, int64_t p, int64_t h0, int layout, uint64_t *acc, void *stream) {

@@ -49,8 +49,26 @@ __global__ void gen_prefix_kernel(uint32_t *dst, long long n, long long p, long 
     }
 }
 
+__device__ __forceinline__ uint32_t tri_full_bits(uint64_t u, long long a, long long b, long long n, int dtype) {
+    // kind 1 ('full', bulkgen/__init__.py): signed weights on every entry Algorithm OPT
+    // reads (b - a >= 2, the root side included), poison on the entries it never reads
+    if (b - a >= 2) {
+        if (dtype == BO_I32) {
+            const long long B = (1LL << 31) / (2 * (n - 2 > 1 ? n - 2 : 1));
+            return static_cast<uint32_t>(static_cast<int32_t>(
+                static_cast<long long>((u >> 32) % static_cast<uint64_t>(2 * B - 1)) - (B - 1)));
+        }
+        return __float_as_uint(static_cast<float>(u >> 40) * 0x1p-23f - 1.0f);
+    }
+    if (dtype == BO_I32) return static_cast<uint32_t>(u >> 32);
+    const uint32_t poison[8] = {0x7FC00000u, 0x7F800000u, 0xFF800000u, 0x7F7FFFFFu,
+                                0xFF7FFFFFu, 0x7FA00000u, 0x80000000u, 0u};
+    const uint32_t q = poison[u >> 61];
+    return q ? q : __float_as_uint(static_cast<float>(u >> 40) * 0x1p-23f - 1.0f);
+}
+
 __global__ void gen_tri_kernel(uint32_t *dst, long long n, long long p, long long h0, uint64_t seed, int dtype,
-                               int layout) {
+                               int layout, int kind) {
     pdl_begin();
     // walks the dense (h, a, b) space; packed layouts store only b - a >= 2
     const long long nn = n * n, total = nn * p;
@@ -62,7 +80,9 @@ __global__ void gen_tri_kernel(uint32_t *dst, long long n, long long p, long lon
         const long long a = e / n, b = e - a * n;
         if (layout >= BO_PACKED_ROW && b - a < 2) continue;
         uint32_t bits = 0;
-        if (b - a >= 2 && !(a == 0 && b == n - 1)) {
+        if (kind == 1) {
+            bits = tri_full_bits(gen_u(seed, static_cast<uint64_t>(h0 + h), static_cast<uint64_t>(e)), a, b, n, dtype);
+        } else if (b - a >= 2 && !(a == 0 && b == n - 1)) {
             const uint64_t u = gen_u(seed, static_cast<uint64_t>(h0 + h), static_cast<uint64_t>(e));
             bits = dtype == BO_I32 ? static_cast<uint32_t>(u >> 44)
                                    : __float_as_uint(static_cast<float>(u >> 40) * 0x1p-24f);
@@ -102,11 +122,11 @@ int launch_gen_prefix(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed
     return after_launch("gen_prefix_kernel");
 }
 
-int launch_gen_tri(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout,
+int launch_gen_tri(void *dst, int64_t n, int64_t p, int64_t h0, uint64_t seed, int dtype, int layout, int kind,
                    cudaStream_t st) {
     if (n * n * p == 0) return BO_OK;
     launch(gen_tri_kernel, grid_for(n * n * p), 256, 0, st, static_cast<uint32_t *>(dst), n, p, h0, seed, dtype,
-                                                        layout);
+                                                        layout, kind);
     return after_launch("gen_tri_kernel");
 }
 

@@ -49,13 +49,14 @@ def test_device_generator_equals_bulkgen(dt, layout, kind):
     assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
 
 
+@pytest.mark.parametrize("kind", ["chords", "full"])
 @pytest.mark.parametrize("dt", ["int32", "float32"])
 @pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE, bo.PACKED_ROW, bo.PACKED_COLUMN])
-def test_device_tri_generator_equals_bulkgen(dt, layout):
-    n, p, h0 = 13, 29, 5
-    got = bo.generate_tri(n, p, 3, getattr(torch, dt), layout, h0=h0).cpu().numpy()
-    ref = bulkgen.tri_input(n, p, 3, dt, layout, h0=h0)
-    assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+def test_device_tri_generator_equals_bulkgen(dt, layout, kind):
+    for n, p, h0 in ((13, 29, 5), (3, 4, 0), (64, 9, 77)):
+        got = bo.generate_tri(n, p, 3, getattr(torch, dt), layout, h0=h0, kind=kind).cpu().numpy()
+        ref = bulkgen.tri_input(n, p, 3, dt, layout, h0=h0, kind=kind)
+        assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
 
 
 def test_checksum_device_equals_host():
@@ -90,9 +91,10 @@ def test_prefix_host_transposed_variant():
 @pytest.mark.parametrize("variant", [bo.AUTO, bo.TRI_UMM_GLOBAL])
 def test_tri_host_entry_point(layout, variant):
     n, p = 16, 2000
-    c = bulkgen.tri_input(n, p, seed=4, dtype="int32", layout=layout)
-    out = bo.triangulation_host(torch.from_numpy(c).pin_memory(), layout, variant)
-    assert np.array_equal(out.numpy(), oracle.bulk_opt(c, layout))
+    for kind in ("chords", "full"):
+        c = bulkgen.tri_input(n, p, seed=4, dtype="int32", layout=layout, kind=kind)
+        out = bo.triangulation_host(torch.from_numpy(c).pin_memory(), layout, variant)
+        assert np.array_equal(out.numpy(), oracle.bulk_opt(c, layout))
 
 
 def test_launch_counter_counts_kernels():
@@ -107,7 +109,7 @@ def test_launch_counter_counts_kernels():
 @pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
 def test_tri_host_entry_point_chunked_variants(n, p, variant, layout):
     # several chunks in flight on the two internal streams; TILED_GLOBAL gives each stream its own scratch
-    c = bulkgen.tri_input(n, p, seed=n + p, dtype="float32", layout=layout)
+    c = bulkgen.tri_input(n, p, seed=n + p, dtype="float32", layout=layout, kind="full")
     dt = bo.F32
     need = bo.triangulation_host_bytes(n, p, dt, layout, variant)
     assert need >= c.size * 4 + p * 4

@@ -207,3 +207,105 @@ def test_every_n_auto(dt, layout):
         ref = oracle.bulk_opt(c, layout, nthreads=NTHREADS)
         got = bo.triangulation(torch.from_numpy(c).to(DEV), layout).cpu().numpy()
         assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), n
+
+
+# ---------------------------------------------------------------------------
+# Un-narrowed inputs ('full' kind, bulkgen): signed weights on every entry
+# Algorithm OPT reads -- the root side c[0][n-1] included, which P:199 adds at
+# i = 1, j = n-1 -- and poison (NaN, +-inf, +-FLT_MAX, -0, garbage int32) on
+# every entry it never reads (sides, diagonal, lower triangle; P:212 stores
+# only b - a >= 2).  Any kernel that drops the root term, or lets an unread
+# entry into its table, fails here.
+# ---------------------------------------------------------------------------
+FULL_CASES = [(3, 9), (4, 33), (5, 40), (7, 65), (8, 100), (12, 50), (13, 129), (16, 300), (17, 64), (18, 40),
+              (21, 35), (24, 100), (29, 33), (33, 64), (40, 70), (47, 20), (56, 19), (57, 17), (61, 33), (63, 33),
+              (64, 130), (65, 20), (66, 9), (100, 9), (128, 4), (131, 3)]
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", LAYOUTS)
+@pytest.mark.parametrize("n,p", FULL_CASES)
+def test_full_inputs_every_variant_matches_oracle(dt, layout, n, p):
+    c = bulkgen.tri_input(n, p, seed=5 * n + p, dtype=dt, layout=layout, kind="full")
+    ref = oracle.bulk_opt(c, layout, nthreads=NTHREADS)
+    ct = torch.from_numpy(c).to(DEV)
+    for v in _variants(n):
+        if not _supported(n, v):
+            continue
+        got = bo.triangulation(ct, layout, v).cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), ref.view(np.uint32)), (n, p, v)
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", LAYOUTS)
+@pytest.mark.parametrize("n,p", [(3, 7), (4, 40), (5, 33), (9, 64), (16, 300), (17, 50), (31, 40), (33, 64),
+                                 (61, 20), (63, 21), (64, 130)])
+def test_full_inputs_chords_match_oracle(dt, layout, n, p):
+    c = bulkgen.tri_input(n, p, seed=3 * n + p, dtype=dt, layout=layout, kind="full")
+    ref_v, ref_ch = oracle.bulk_opt_chords(c, layout)
+    v, ch = bo.triangulation_chords(torch.from_numpy(c).to(DEV), layout)
+    assert np.array_equal(v.cpu().numpy().view(np.uint32), ref_v.view(np.uint32))
+    assert np.array_equal(ch.cpu().numpy(), ref_ch)
+
+
+def test_full_inputs_root_side_is_added():
+    # the same instances with c[0][n-1] zeroed: every GPU result moves by exactly the root weight
+    for n, dt in ((16, torch.int32), (40, torch.int32), (64, torch.int32), (130, torch.int32)):
+        c = bo.generate_tri(n, 500, 21, dt, bo.ROW_WISE, kind="full")
+        d = c.clone()
+        d[:, 0, n - 1] = 0
+        for v in _variants(n):
+            if _supported(n, v):
+                got = bo.triangulation(c, bo.ROW_WISE, v).long()
+                z = bo.triangulation(d, bo.ROW_WISE, v).long()
+                assert torch.equal(got - z, c[:, 0, n - 1].long()), (n, v)
+
+
+def test_full_inputs_unread_entries_are_never_read():
+    # re-poisoning the unread entries with other values changes nothing, bit for bit
+    for n in (7, 16, 33, 64, 80):
+        c = bo.generate_tri(n, 700, 22, torch.float32, bo.ROW_WISE, kind="full")
+        a_ = torch.arange(n, device=DEV)
+        unread = (a_[None, :] - a_[:, None] < 2)
+        d = c.clone()
+        d[:, unread] = float("-inf")
+        e = c.clone()
+        e[:, unread] = float("nan")
+        for v in _variants(n):
+            if _supported(n, v):
+                r = bo.triangulation(c, bo.ROW_WISE, v).view(torch.int32)
+                assert torch.equal(r, bo.triangulation(d, bo.ROW_WISE, v).view(torch.int32)), (n, v)
+                assert torch.equal(r, bo.triangulation(e, bo.ROW_WISE, v).view(torch.int32)), (n, v)
+
+
+# Table-slot reuse: with p large enough every persistent CTA (tiled kernels) or
+# workspace slot (CTA-per-instance kernels) runs several instances in turn, so
+# cells left by instance h -- including the padding columns b >= n when n % 4 != 0
+# -- are live in the table when instance h + stride starts.
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("n,p", [(17, 200000), (18, 150000), (33, 60000), (41, 40000), (61, 12000), (63, 12000),
+                                 (65, 1200), (130, 500)])
+def test_multipass_table_reuse_full_inputs(dt, n, p):
+    c = bo.generate_tri(n, p, 23 + n, getattr(torch, dt), bo.ROW_WISE, kind="full")
+    ids = np.arange(p) if n <= 33 or NTHREADS >= 16 else np.unique(np.r_[np.arange(0, p, 7), p - 1])
+    ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 23 + n, dt, kind="full"), oracle.ROW_WISE,
+                          nthreads=NTHREADS)
+    for v in _variants(n):
+        if v == bo.TRI_UMM_GLOBAL and n > 64:
+            continue                                    # (n-1)^2 p workspace; covered above at small p
+        if _supported(n, v):
+            got = bo.triangulation(c, bo.ROW_WISE, v).cpu().numpy()
+            assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32)), (n, v)
+
+
+@pytest.mark.parametrize("layout", LAYOUTS)
+def test_full_inputs_tr1_tr2_shapes(layout):
+    # the configs' shapes on un-narrowed inputs: TR-1 (int32 n=16) on every instance,
+    # TR-2 (fp32 n=64) on every 8th instance + the last
+    for n, p, dt, step in ((16, 65536, "int32", 1), (64, 65536, "float32", 8)):
+        c = bo.generate_tri(n, p, 24, getattr(torch, dt), layout, kind="full")
+        got = bo.triangulation(c, layout).cpu().numpy()
+        ids = np.unique(np.r_[np.arange(0, p, step), p - 1])
+        ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 24, dt, kind="full"), oracle.ROW_WISE,
+                              nthreads=NTHREADS)
+        assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32)), (n, layout)

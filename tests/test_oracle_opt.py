@@ -256,3 +256,58 @@ def test_packed_index_closed_form():
         assert k == a * (n - 2) - a * (a - 1) // 2 + (b - a - 2)
     # every weight Algorithm OPT reads appears exactly once (trace test: {b-a >= 2})
     assert sorted(pairs) == sorted((a, b) for a in range(n) for b in range(a + 2, n))
+
+
+# ------------------------------------------- 'full' inputs (every entry non-zero)
+# Algorithm OPT reads c[i-1, j] for 1 <= i < j <= n-1 only, i.e. the
+# entries b - a >= 2, the root side c[0][n-1] among them (reading G8).  The
+# 'full' generator puts signed weights there and poison (NaN, +-inf, +-FLT_MAX,
+# -0, garbage int32) everywhere else; the pins below fix what the result must be.
+def _zero_unread(c):
+    n = c.shape[-1]
+    a = np.arange(n)[:, None]
+    b = np.arange(n)[None, :]
+    return np.where(b - a >= 2, c, np.zeros((), dtype=c.dtype))
+
+
+@pytest.mark.parametrize("n", range(3, 11))
+def test_full_kind_int32_equals_brute_force_with_root(n):
+    for h in range(5 if n < 10 else 2):
+        c = bulkgen.tri_instances(n, [h], seed=300 + n, dtype="int32", kind="full")[0]
+        assert c[0, n - 1] != 0
+        bv, _ = oracle.brute_opt(_zero_unread(c))      # brute force adds c[0][n-1]
+        assert oracle.opt(c) == int(bv)
+
+
+@pytest.mark.parametrize("n", range(3, 10))
+def test_full_kind_fp32_within_rounding_of_brute_force(n):
+    for h in range(4):
+        c = bulkgen.tri_instances(n, [h], seed=400 + n, dtype="float32", kind="full")[0]
+        bv, _ = oracle.brute_opt(_zero_unread(c))
+        v = float(oracle.opt(c))
+        # signed weights in [-1, 1): n-2 terms, each fp32 add errs <= 2^-24 * |partial| <= 2^-24 (n-2)
+        assert abs(v - bv) <= (n - 2) ** 2 * 2.0 ** -24
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("n", [3, 4, 7, 16, 33, 64])
+def test_unread_entries_never_reach_the_result(dt, n):
+    c = bulkgen.tri_input(n, 40, seed=9, dtype=dt, kind="full")
+    ref = oracle.bulk_opt(_zero_unread(c), oracle.ROW_WISE)
+    got = oracle.bulk_opt(c, oracle.ROW_WISE)
+    assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+    # and the root side does: Algorithm OPT adds c[0][n-1] last
+    d = c.copy()
+    d[:, 0, n - 1] = 0
+    delta = got.astype(np.float64) - oracle.bulk_opt(d, oracle.ROW_WISE).astype(np.float64)
+    if dt == "int32":
+        assert np.array_equal(delta, c[:, 0, n - 1].astype(np.float64))
+    else:
+        assert np.allclose(delta, c[:, 0, n - 1], atol=n * 2.0 ** -22)
+
+
+def test_full_kind_root_shift_closed_form_n4():
+    # n = 4: two triangulations; OPT = min(c[0][2], c[1][3]) + c[0][3] with signed weights
+    c = bulkgen.tri_instances(4, np.arange(200), seed=5, dtype="int32", kind="full")
+    for x in c:
+        assert oracle.opt(x) == min(int(x[0, 2]), int(x[1, 3])) + int(x[0, 3])

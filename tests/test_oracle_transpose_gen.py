@@ -62,3 +62,26 @@ def test_checksum_is_layout_and_order_independent():
     # shards sum to the whole (mod 2^64)
     s = (bulkgen.checksum(x[:3]) + bulkgen.checksum(x[3:], h0=3)) % 2**64
     assert s == a
+
+
+@pytest.mark.parametrize("n", [3, 5, 16, 64, 130])
+def test_full_tri_generator_structure(n):
+    ci = bulkgen.tri_instances(n, np.arange(50), seed=6, dtype="int32", kind="full")
+    cf = bulkgen.tri_instances(n, np.arange(50), seed=6, dtype="float32", kind="full")
+    a = np.arange(n)[:, None]
+    b = np.arange(n)[None, :]
+    read = np.broadcast_to(b - a >= 2, ci.shape)
+    B = bulkgen.tri_int32_bound(n)
+    assert B * 2 * (n - 2) <= 2 ** 31 < (B + 1) * 2 * (n - 2)
+    assert np.abs(ci[read].astype(np.int64)).max() <= B - 1
+    assert (ci[read] < 0).any() and (ci[:, 0, n - 1] != 0).all()
+    assert np.isfinite(cf[read]).all() and cf[read].min() >= -1 and cf[read].max() < 1 and (cf[read] < 0).any()
+    if n >= 5:
+        unread = cf[~read]
+        assert np.isnan(unread).any() and np.isinf(unread).any() and (np.abs(unread) == np.finfo(np.float32).max).any()
+    # chords kind unchanged by the kind argument's default
+    assert np.array_equal(bulkgen.tri_instances(n, [1], 6, "int32"), bulkgen.tri_instances(n, [1], 6, "int32", "chords"))
+    # layouts: packed keeps exactly the read entries
+    pk = bulkgen.tri_input(n, 50, seed=6, dtype="float32", layout=bulkgen.PACKED_ROW, kind="full")
+    pr = bulkgen.packed_pairs(n)
+    assert np.array_equal(pk.view(np.uint32), cf[:, [x for x, _ in pr], [y for _, y in pr]].view(np.uint32))
