@@ -82,13 +82,14 @@ typedef enum {
                                wavefront, k split across lanes + shuffle min      */
     BO_TRI_THREAD_REG = 18, /* thread per instance, M in registers (3 <= n <= 18) */
     BO_TRI_TILED = 19,      /* warp per instance, M in shared memory, 4x4 register
-                               tiles (min-plus blocked product), 5 <= n <= 64     */
+                               tiles (min-plus blocked product), 3 <= n <= 64     */
     BO_TRI_TILED_HALF = 20, /* as BO_TRI_TILED with 16 lanes per instance (two
                                instances per warp)                                 */
     BO_TRI_TILED_GLOBAL = 21, /* CTA per instance, same blocked algorithm, table in a
                                per-CTA global workspace slot kept L2-resident
                                (AUTO for 64 < n < 512); workspace
-                               min(p, #SMs) * 16 * (2T^2 + 3T) bytes, T = ceil(n/4) */
+                               min(p, #SMs) * 16 * (2T^2 + 3T) bytes, T = ceil(n/4),
+                               16-byte aligned                                    */
     BO_TRI_TILED_QUARTER = 22, /* as BO_TRI_TILED with 8 lanes per instance (four
                                instances per warp; a lane takes several tiles of a
                                tile-diagonal in turn)                             */
@@ -133,8 +134,14 @@ size_t bulk_prefix_sums_workspace(int64_t n, int64_t p, int dtype, int layout, i
 /*   |c| < FLT_MAX / (2(n-2)) (no sum overflows).  Results are then           */
 /*   bit-identical to the sequential algorithm: min is exact, every sum keeps */
 /*   its association, and no table value is ever -0 (reading G16). */
-/*   workspace: device, >= bulk_triangulation_workspace(...) bytes (only      */
-/*   BO_TRI_UMM_GLOBAL needs one).                                            */
+/*   workspace: device, >= bulk_triangulation_workspace(...) bytes; NULL is   */
+/*   fine when that is 0.  Needed by BO_TRI_UMM_GLOBAL, BO_TRI_TILED_GLOBAL   */
+/*   (16-byte aligned) and BO_TRI_TILED_GLOBAL8 (32-byte aligned), hence by   */
+/*   BO_AUTO for every n > 64.  Misaligned or short: BO_EINVAL.  One         */
+/*   workspace must not be shared by launches in flight on different streams.*/
+/*   Variant n ranges: THREAD_REG 3..18, TILED / TILED_HALF / TILED_QUARTER  */
+/*   3..64, SMEM_WARP while one table fits in 200 KB of shared memory,        */
+/*   TILED_GLOBAL / GLOBAL8 / UMM_GLOBAL 3..4096; otherwise BO_EUNSUPPORTED.  */
 /* ------------------------------------------------------------------------- */
 int bulk_triangulation(const void *c, void *out, int64_t n, int64_t p, int dtype, int layout,
                        int variant, void *workspace, size_t workspace_bytes, void *stream);

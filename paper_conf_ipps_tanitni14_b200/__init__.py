@@ -120,6 +120,20 @@ def _need_cuda(*ts):
             raise ValueError("tensors must be contiguous")
 
 
+def _check_out(out: torch.Tensor, like: torch.Tensor, shape, what: str = "out"):
+    """The C ABI cannot see buffer sizes: a caller-supplied output must be a
+    contiguous CUDA tensor on the input's device, of its dtype and `shape`."""
+    _need_cuda(out)
+    if out.device != like.device or out.dtype != like.dtype or tuple(out.shape) != tuple(shape):
+        raise ValueError(f"{what} must be a {like.dtype} tensor of shape {tuple(shape)} on {like.device}")
+
+
+def _check_workspace(ws: torch.Tensor, like: torch.Tensor):
+    _need_cuda(ws)
+    if ws.device != like.device:
+        raise ValueError(f"workspace must be on {like.device}")
+
+
 def _shape_np(t: torch.Tensor, layout: int):
     if t.dim() != 2:
         raise ValueError("prefix sums take a 2-D tensor: [p, n] row-wise or [n, p] column-wise")
@@ -140,12 +154,13 @@ def prefix_sums(x: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, ou
     dt = _dtype_code(x)
     if out is None:
         out = torch.empty_like(x)
-    _need_cuda(out)
+    _check_out(out, x, x.shape)
     need = prefix_sums_workspace(n, p, dt, layout, variant)
     wptr, wbytes = None, 0
     if need:
         if workspace is None:
             workspace = torch.empty(need, dtype=torch.uint8, device=x.device)
+        _check_workspace(workspace, x)
         wptr, wbytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
     _check(lib().bulk_prefix_sums(x.data_ptr(), out.data_ptr(), n, p, dt, layout, variant, wptr, wbytes,
                                   _stream(stream, x)))
@@ -220,11 +235,13 @@ def triangulation(c: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, 
     dt = _dtype_code(c)
     if out is None:
         out = torch.empty(p, dtype=c.dtype, device=c.device)
+    _check_out(out, c, (p,))
     need = triangulation_workspace(n, p, dt, layout, variant)
     wptr, wbytes = None, 0
     if need:
         if workspace is None:
             workspace = torch.empty(need, dtype=torch.uint8, device=c.device)
+        _check_workspace(workspace, c)
         wptr, wbytes = workspace.data_ptr(), workspace.numel() * workspace.element_size()
     _check(lib().bulk_triangulation(c.data_ptr(), out.data_ptr(), n, p, dt, layout, variant, wptr, wbytes,
                                     _stream(stream, c)))
@@ -242,9 +259,10 @@ def triangulation_chords(c: torch.Tensor, layout: int = ROW_WISE, stream=None, o
         out = torch.empty(p, dtype=c.dtype, device=c.device)
     if chords is None:
         chords = torch.empty((p, max(n - 3, 0), 2), dtype=torch.int16, device=c.device)
-    _need_cuda(out, chords)
-    if out.dtype != c.dtype or out.numel() != p or chords.dtype != torch.int16 or chords.numel() != p * max(n - 3, 0) * 2:
-        raise ValueError("out must be [p] of the weights' dtype and chords [p, n-3, 2] int16")
+    _check_out(out, c, (p,))
+    _need_cuda(chords)
+    if chords.device != c.device or chords.dtype != torch.int16 or chords.numel() != p * max(n - 3, 0) * 2:
+        raise ValueError("chords must be [p, n-3, 2] int16 on the weights' device")
     _check(lib().bulk_triangulation_chords(c.data_ptr(), out.data_ptr(), chords.data_ptr() if chords.numel() else None,
                                            n, p, dt, layout, _stream(stream, c)))
     return out, chords
@@ -295,6 +313,7 @@ def transpose(x: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> 
     rows, cols = x.shape
     if out is None:
         out = torch.empty((cols, rows), dtype=x.dtype, device=x.device)
+    _check_out(out, x, (cols, rows))
     _check(lib().bulk_transpose(x.data_ptr(), out.data_ptr(), rows, cols, 4, _stream(stream, x)))
     return out
 

@@ -6,6 +6,7 @@
 #include <cstring>
 #include <mutex>
 #include <set>
+#include <thread>
 #include <string>
 #include <utility>
 #include <vector>
@@ -62,6 +63,42 @@ bool ensure_dyn_smem(const void *func, int bytes) {
     if (cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess) return false;
     done.insert(key);
     return true;
+}
+
+int work_slot_for(cudaStream_t st) {
+    // A queue slot is reset by the last CTA of the launch that used it, so two
+    // launches may share one only if the second cannot start before the first
+    // has finished: launches on one stream (griddepcontrol.wait precedes every
+    // access to the slot).  So each (device, stream) owns a slot.  A launch
+    // being captured into a graph gets none (-1: static tile striding): the
+    // graph may be replayed on any stream, beside eager launches on this one.
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(st, &cap) != cudaSuccess) {
+        cudaGetLastError();
+        return -1;
+    }
+    if (cap != cudaStreamCaptureStatusNone) return -1;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    // cudaStreamPerThread is one handle for a different stream in every thread
+    const std::thread::id tid = st == cudaStreamPerThread ? std::this_thread::get_id() : std::thread::id();
+    struct Owner {
+        int dev;
+        cudaStream_t st;
+        std::thread::id tid;
+    };
+    static std::mutex mu;
+    static std::vector<Owner> owners;                            // in order of first use
+    std::lock_guard<std::mutex> g(mu);
+    int used_on_dev = 0;
+    for (const Owner &o : owners) {
+        if (o.dev != dev) continue;
+        if (o.st == st && o.tid == tid) return used_on_dev;
+        ++used_on_dev;
+    }
+    if (used_on_dev >= kWorkSlots) return -1;                   // beyond 256 streams: static striding
+    owners.push_back(Owner{dev, st, tid});
+    return used_on_dev;
 }
 
 // ---------------------------------------------------------------- TMA maps
@@ -147,6 +184,11 @@ static bool ranges_partially_overlap(const void *a, const void *b, size_t bytes)
     return x < y + bytes && y < x + bytes;
 }
 
+static bool ranges_intersect(const void *a, size_t abytes, const void *b, size_t bbytes) {
+    const uintptr_t x = reinterpret_cast<uintptr_t>(a), y = reinterpret_cast<uintptr_t>(b);
+    return x < y + bbytes && y < x + abytes;
+}
+
 static int check_prefix_args(const void *src, const void *dst, int64_t n, int64_t p, int dtype, int layout,
                              int variant) {
     if (n < 0 || p < 0) return fail(BO_EINVAL, "prefix: n and p must be >= 0");
@@ -191,7 +233,11 @@ static size_t prefix_ws(int64_t n, int64_t p, int variant) {
 }
 
 // Internal streams for the host-buffer pipeline (one pair per device).
+// `mu` is held from the ev_start record to the caller's final waits, so two
+// host threads never interleave chunks on the internal streams or re-record
+// ev_start between another call's record and its waits.
 struct HostPipe {
+    std::mutex mu;
     cudaStream_t s[2] = {nullptr, nullptr};
     cudaEvent_t ev_start = nullptr, ev_done[2] = {nullptr, nullptr};
 };
@@ -254,7 +300,9 @@ int bulk_prefix_sums(const void *src, void *dst, int64_t n, int64_t p, int dtype
     const size_t need = prefix_ws(n, p, v);
     if (need > 0 && (!workspace || workspace_bytes < need))
         return fail(BO_EINVAL, "prefix: workspace too small (need " + std::to_string(need) + " bytes)");
-    if (need > 0 && (ranges_partially_overlap(workspace, src, need) || workspace == src || workspace == dst))
+    // the workspace (need bytes) must share no byte with src or dst (n*p*4 bytes each)
+    if (need > 0 && (ranges_intersect(workspace, need, src, static_cast<size_t>(n * p) * 4) ||
+                     ranges_intersect(workspace, need, dst, static_cast<size_t>(n * p) * 4)))
         return fail(BO_EINVAL, "prefix: workspace overlaps the data");
     return prefix_dispatch(src, dst, n, p, dtype, layout, v, workspace, static_cast<cudaStream_t>(stream));
 }
@@ -387,6 +435,7 @@ int bulk_prefix_sums_host(const void *h_src, void *h_dst, int64_t n, int64_t p, 
                                    std::to_string(data_bytes + 2 * ws_chunk) + " bytes)");
     HostPipe *hp = host_pipe();
     cudaStream_t caller = static_cast<cudaStream_t>(stream);
+    std::unique_lock<std::mutex> pipe_lock(hp->mu);
     if ((rc = cuda_check(cudaEventRecord(hp->ev_start, caller), "prefix_host: event"))) return rc;
     for (int i = 0; i < 2; ++i)
         if ((rc = cuda_check(cudaStreamWaitEvent(hp->s[i], hp->ev_start, 0), "prefix_host: wait"))) return rc;
@@ -423,6 +472,7 @@ int bulk_prefix_sums_host(const void *h_src, void *h_dst, int64_t n, int64_t p, 
         if ((rc = cuda_check(cudaEventRecord(hp->ev_done[i], hp->s[i]), "prefix_host: event"))) return rc;
         if ((rc = cuda_check(cudaStreamWaitEvent(caller, hp->ev_done[i], 0), "prefix_host: wait"))) return rc;
     }
+    pipe_lock.unlock();
     return cuda_check(cudaStreamSynchronize(caller), "prefix_host: sync");
 }
 
@@ -458,6 +508,7 @@ int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, 
                                    std::to_string(ws_off + ws_bytes) + " bytes)");
     HostPipe *hp = host_pipe();
     cudaStream_t caller = static_cast<cudaStream_t>(stream);
+    std::unique_lock<std::mutex> pipe_lock(hp->mu);
     if ((rc = cuda_check(cudaEventRecord(hp->ev_start, caller), "tri_host: event"))) return rc;
     for (int i = 0; i < 2; ++i)
         if ((rc = cuda_check(cudaStreamWaitEvent(hp->s[i], hp->ev_start, 0), "tri_host: wait"))) return rc;
@@ -491,6 +542,7 @@ int bulk_triangulation_host(const void *h_c, void *h_out, int64_t n, int64_t p, 
         if ((rc = cuda_check(cudaEventRecord(hp->ev_done[i], hp->s[i]), "tri_host: event"))) return rc;
         if ((rc = cuda_check(cudaStreamWaitEvent(caller, hp->ev_done[i], 0), "tri_host: wait"))) return rc;
     }
+    pipe_lock.unlock();
     return cuda_check(cudaStreamSynchronize(caller), "tri_host: sync");
 }
 

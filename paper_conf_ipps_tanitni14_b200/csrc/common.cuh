@@ -161,19 +161,25 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
 // Dynamic tile scheduler for persistent kernels: CTA b starts on tile b, then
 // claims gridDim.x + (ticket) until the tiles run out, so SMs that run faster
 // (L2 die, DRAM channel mix) take more tiles.  The last CTA to retire resets
-// the slot, so no host memset is needed between launches; the host rotates
-// through kWorkSlots slots so launches on different streams do not share one.
+// the slot, so no host memset is needed between launches.  The host gives each
+// (device, stream) its own slot (work_slot_for, api.cu), and none (-1) to a
+// launch being captured into a graph: with no slot the CTAs stride statically
+// (tile b, b + gridDim.x, ...), so no two grids can ever share a counter.
 struct WorkSlot {
     unsigned long long next;
     unsigned int done;
     unsigned int pad;
 };
 constexpr int kWorkSlots = 256;
+int work_slot_for(cudaStream_t st);
 
-__device__ __forceinline__ long long claim_tile(WorkSlot *w) {
+// next tile after `cur` for this CTA: dynamic (w != nullptr) or static striding
+__device__ __forceinline__ long long claim_tile(WorkSlot *w, long long cur) {
+    if (w == nullptr) return cur + static_cast<long long>(gridDim.x);
     return static_cast<long long>(gridDim.x) + static_cast<long long>(atomicAdd(&w->next, 1ull));
 }
 __device__ __forceinline__ void retire_cta(WorkSlot *w) {
+    if (w == nullptr) return;
     __threadfence();
     if (atomicAdd(&w->done, 1u) == gridDim.x - 1) {
         w->next = 0;

@@ -111,12 +111,6 @@ template <int INST> struct Cfg {
 }  // namespace fr
 
 __device__ WorkSlot g_fr_slots[kWorkSlots];
-// one allocator for every kernel that draws on g_fr_slots: launches in flight
-// at the same time (other streams) must never share a queue slot
-static int fr_next_slot() {
-    static std::atomic<unsigned> next{0};
-    return static_cast<int>(next.fetch_add(1) % kWorkSlots);
-}
 
 template <typename T, int kInst>
 __global__ void __launch_bounds__(kInst)
@@ -132,7 +126,7 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
     uint64_t *full = reinterpret_cast<uint64_t *>(buf + kStages * kBoxBytes);
     int *stage_tile = reinterpret_cast<int *>(full + kStages);    // tile of each ring slot, -1 = end
     int *stage_chunk = stage_tile + kStages;
-    WorkSlot *ws = &g_fr_slots[slot];
+    WorkSlot *ws = slot >= 0 ? &g_fr_slots[slot] : nullptr;
     const int tid = threadIdx.x;
 
     if (tid == 0) {
@@ -149,7 +143,7 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
     bool prod_done = false;
     auto issue = [&](int s) {
         if (prod_chunk == nchunks) {
-            prod_tile = claim_tile(ws);
+            prod_tile = claim_tile(ws, prod_tile);
             prod_chunk = 0;
         }
         if (prod_tile >= ntiles) {
@@ -239,7 +233,7 @@ ps_across_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant
     uint64_t *full = reinterpret_cast<uint64_t *>(buf + kStages * kBoxBytes);
     int *stage_tile = reinterpret_cast<int *>(full + kStages);
     int *stage_chunk = stage_tile + kStages;
-    WorkSlot *ws = &g_fr_slots[slot];
+    WorkSlot *ws = slot >= 0 ? &g_fr_slots[slot] : nullptr;
     const int tid = threadIdx.x;
     if (tid == 0) {
         prefetch_tmap(&src_map);
@@ -253,7 +247,7 @@ ps_across_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant
     bool prod_done = false;
     auto issue = [&](int s) {
         if (prod_chunk == nchunks) {
-            prod_tile = claim_tile(ws);
+            prod_tile = claim_tile(ws, prod_tile);
             prod_chunk = 0;
         }
         if (prod_tile >= ntiles) {
@@ -431,7 +425,7 @@ static int launch_across_tma(const T *src, T *dst, int64_t n, int64_t p, cudaStr
     int per_sm = 1;
     per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&ps_across_tma<T, INST>), INST, C::kSmem);
     const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
-    const int slot = fr_next_slot();
+    const int slot = work_slot_for(st);
     launch(ps_across_tma<T, INST>, static_cast<unsigned>(grid), INST, C::kSmem, st, smap, dmap, ntiles, nchunks, slot);
     return after_launch("ps_across_tma");
 }
@@ -478,7 +472,7 @@ static int launch_fused_row_tma(const T *src, T *dst, int64_t n, int64_t p, cuda
     int per_sm = 1;
     per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&ps_fused_row_tma<T, INST>), INST, C::kSmem);
     const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
-    const int slot = fr_next_slot();
+    const int slot = work_slot_for(st);
     launch(ps_fused_row_tma<T, INST>, static_cast<unsigned>(grid), INST, C::kSmem, st, smap, dmap, ntiles, nchunks,
                                                                                    slot);
     return after_launch("ps_fused_row_tma");

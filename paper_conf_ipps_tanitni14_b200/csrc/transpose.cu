@@ -44,7 +44,7 @@ transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
     uint8_t *out_buf = base + kStages * kBoxBytes;            // kOut boxes (2 sub-tiles each)
     uint64_t *full = reinterpret_cast<uint64_t *>(out_buf + kOut * kBoxBytes);
     long long *stage_tile = reinterpret_cast<long long *>(full + kStages);   // -1 = end
-    WorkSlot *ws = &g_tr_slots[slot];
+    WorkSlot *ws = slot >= 0 ? &g_tr_slots[slot] : nullptr;
 
     const int tid = threadIdx.x;
     const int warp = tid >> 5, lane = tid & 31;
@@ -67,7 +67,7 @@ transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
             mbar_arrive(&full[s]);
             return;
         }
-        next_tile = claim_tile(ws);
+        next_tile = claim_tile(ws, next_tile);
         stage_tile[s] = t;
         const int tc = static_cast<int>(t % tiles_c), trow = static_cast<int>(t / tiles_c);
         mbar_arrive_expect_tx(&full[s], kBoxBytes);
@@ -158,8 +158,7 @@ int launch_transpose(const void *src, void *dst, int64_t rows, int64_t cols, cud
         int per_sm = 1;
         per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&transpose_tma_kernel), tr::kThreads, tr::kSmem);
         const long long grid = std::min<long long>(ntiles, static_cast<long long>(std::max(per_sm, 1)) * num_sms());
-        static std::atomic<unsigned> next_slot{0};
-        const int slot = static_cast<int>(next_slot.fetch_add(1) % kWorkSlots);
+        const int slot = work_slot_for(st);
         launch(transpose_tma_kernel, static_cast<unsigned>(grid), tr::kThreads, tr::kSmem, st, 
             smap, dmap, static_cast<int>(tiles_c), ntiles, slot);
         return after_launch("transpose_tma_kernel");

@@ -476,7 +476,7 @@ static int run_tri(const void *c, void *out, int64_t n, int64_t p, int layout, i
         case BO_TRI_TILED:
         case BO_TRI_TILED_HALF:
         case BO_TRI_TILED_QUARTER:
-            if (!tiled_supported(n)) return fail(BO_EUNSUPPORTED, "triangulation TILED supports 5 <= n <= 64");
+            if (!tiled_supported(n)) return fail(BO_EUNSUPPORTED, "triangulation TILED supports 3 <= n <= 64");
             return launch_tri_tiled(c, out, n, p, std::is_same<T, float>::value ? BO_F32 : BO_I32, layout,
                                     variant == BO_TRI_TILED ? 32 : variant == BO_TRI_TILED_HALF ? 16 : 8, st);
         case BO_TRI_TILED_GLOBAL:

@@ -835,6 +835,8 @@ size_t tiled_global_workspace(int64_t n, int64_t p) {
 
 int launch_tri_tiled_global(const void *c, void *out, void *ws, int64_t n, int64_t p, int dtype, int layout,
                             cudaStream_t st) {
+    // the kernel moves table rows with 16-byte vector loads and stores
+    if ((reinterpret_cast<uintptr_t>(ws) & 15u) != 0) return fail(BO_EINVAL, "TILED_GLOBAL: workspace must be 16-byte aligned");
     const int NT = static_cast<int>((n + 3) / 4);
     const long long grid = std::min<long long>(p, num_sms());
     const int threads = tiled_global_threads(n);

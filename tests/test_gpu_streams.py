@@ -103,3 +103,66 @@ def test_cuda_graph_capture_and_replay():
     for o, r in zip(outs, ref_x):
         assert torch.equal(o, r)
     assert torch.equal(out_c, ref_c)
+
+
+def test_graph_of_queue_kernels_beside_eager_launches():
+    # the persistent fused-row / column-wise / transpose kernels claim tiles from a
+    # device counter.  A captured launch takes no counter (static tile striding), eager launches
+    # own one per stream, so replaying a graph of those kernels while eager launches of the same
+    # kernels run on another stream can neither skip nor repeat a tile.
+    n, p = 1024, 40000                                   # 128-instance fused-row kernel (dynamic queue)
+    xs = [bo.generate_prefix(n, p, 60 + k, torch.float32, bo.ROW_WISE) for k in range(3)]
+    xc = bo.generate_prefix(256, 40000, 64, torch.int32, bo.COLUMN_WISE)   # column-wise TMA ring
+    ref = [bo.prefix_sums(x, bo.ROW_WISE) for x in xs]
+    ref_c = bo.prefix_sums(xc, bo.COLUMN_WISE)
+    ref_t = bo.transpose(xs[0])
+    torch.cuda.synchronize()
+    cap = torch.cuda.Stream()
+    outs = [torch.empty_like(x) for x in xs]
+    out_c = torch.empty_like(xc)
+    out_t = torch.empty_like(ref_t)
+    with torch.cuda.stream(cap):                          # warm-up on the capture stream
+        for x, o in zip(xs, outs):
+            bo.prefix_sums(x, bo.ROW_WISE, out=o, stream=cap)
+    cap.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=cap):
+        for x, o in zip(xs, outs):
+            bo.prefix_sums(x, bo.ROW_WISE, out=o, stream=cap)
+        bo.prefix_sums(xc, bo.COLUMN_WISE, out=out_c, stream=cap)
+        bo.transpose(xs[0], out=out_t, stream=cap)
+    eager = torch.cuda.Stream()
+    e_outs = [torch.empty_like(x) for x in xs]
+    for rep in range(4):
+        for o in outs + e_outs:
+            o.zero_()
+        out_c.zero_()
+        out_t.zero_()
+        torch.cuda.synchronize()
+        g.replay()                                       # on the current stream
+        with torch.cuda.stream(eager):                   # overlapping eager launches, same kernels
+            for x, o in zip(xs, e_outs):
+                bo.prefix_sums(x, bo.ROW_WISE, out=o, stream=eager)
+            bo.prefix_sums(xc, bo.COLUMN_WISE, stream=eager)
+            bo.transpose(xs[0], stream=eager)
+        torch.cuda.synchronize()
+        for k in range(len(xs)):
+            assert torch.equal(outs[k].view(torch.int32), ref[k].view(torch.int32)), (rep, k)
+            assert torch.equal(e_outs[k].view(torch.int32), ref[k].view(torch.int32)), (rep, k)
+        assert torch.equal(out_c, ref_c), rep
+        assert torch.equal(out_t.view(torch.int32), ref_t.view(torch.int32)), rep
+
+
+def test_out_tensor_is_validated():
+    x = bo.generate_prefix(64, 100, 1, torch.float32, bo.ROW_WISE)
+    with pytest.raises(ValueError):
+        bo.prefix_sums(x, bo.ROW_WISE, out=torch.empty(64 * 99, dtype=torch.float32, device=DEV).view(99, 64))
+    with pytest.raises(ValueError):
+        bo.prefix_sums(x, bo.ROW_WISE, out=torch.empty_like(x, dtype=torch.int32))
+    with pytest.raises(ValueError):
+        bo.prefix_sums(x, bo.ROW_WISE, out=torch.empty(100, 64))           # host tensor
+    c = bo.generate_tri(16, 50, 2, torch.int32, bo.ROW_WISE)
+    with pytest.raises(ValueError):
+        bo.triangulation(c, bo.ROW_WISE, out=torch.empty(49, dtype=torch.int32, device=DEV))
+    with pytest.raises(ValueError):
+        bo.triangulation(c, bo.ROW_WISE, out=torch.empty(50, dtype=torch.float32, device=DEV))

@@ -124,6 +124,54 @@ __global__ void __launch_bounds__(128) i32_addmin_xor(int *out, int iters, int s
     if (s == 12345) out[0] = s;
 }
 
+
+// Single-pipe probes: what each half of the fp32 mix reaches on its own pipe
+// (FADD2 -> FMA pipe, FMNMX3 -> ALU pipe), 16 independent chains per thread.
+// If each alone runs its pipe at ~100 %, the mix's ceiling is the dual-pipe one:
+// one FADD2 (2 adds) + one FMNMX3 (2 mins) per lane per 2 cycles per SMSP =
+// 128 add-mins per SM per clock; the mix kernel above shows how close the
+// kernel's own instruction pairing gets.
+__global__ void __launch_bounds__(128) fp32_fadd2_only(float *out, int iters, float seed) {
+    float2 x[16];
+    const float2 k = make_float2(seed, seed * 0.5f);
+#pragma unroll
+    for (int i = 0; i < 16; ++i) x[i] = make_float2(seed + i + threadIdx.x, seed - i);
+#pragma unroll 1
+    for (int it = 0; it < iters; ++it) {
+#pragma unroll
+        for (int r = 0; r < 16; ++r)
+#pragma unroll
+            for (int i = 0; i < 16; ++i) x[i] = __fadd2_rn(x[i], k);
+    }
+    float s = 0;
+#pragma unroll
+    for (int i = 0; i < 16; ++i) s += x[i].x + x[i].y;
+    if (s == 1.2345f) out[0] = s;
+}
+__global__ void __launch_bounds__(128) fp32_fmnmx3_only(float *out, int iters, float seed) {
+    float x[16], y[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) x[i] = seed + i + threadIdx.x, y[i] = seed * i;
+#pragma unroll 1
+    for (int it = 0; it < iters; ++it) {
+#pragma unroll
+        for (int r = 0; r < 16; ++r)
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+                // x[i] = min(x[i], y[i], y[i+1]); y[i] = max(...) keeps the values moving
+                x[i] = fminf(fminf(x[i], y[i]), y[(i + 1) & 15]);
+                if (i == 15) {
+#pragma unroll
+                    for (int j = 0; j < 16; ++j) y[j] = x[(j + r) & 15];
+                }
+            }
+    }
+    float s = 0;
+#pragma unroll
+    for (int i = 0; i < 16; ++i) s += x[i];
+    if (s == 1.2345f) out[0] = s;
+}
+
 int main(int argc, char **argv) {
     const bool once = argc > 1 && !strcmp(argv[1], "--once");     // one launch of each (for ncu)
     int sms = 0, clk_khz = 0;
@@ -151,7 +199,18 @@ int main(int argc, char **argv) {
             i32_addmin_xor<<<blocks, threads>>>(io, iters, 3);
             cudaEventRecord(b); cudaEventSynchronize(b); cudaEventElapsedTime(&ms, a, b);
             const double ix = double(blocks) * threads * per_thread / (ms * 1e-3);
+            cudaEventRecord(a);
+            fp32_fadd2_only<<<blocks, threads>>>(fo, iters, 1.5f);
+            cudaEventRecord(b); cudaEventSynchronize(b); cudaEventElapsedTime(&ms, a, b);
+            const double fa = double(blocks) * threads * double(iters) * 256 * 2 / (ms * 1e-3);   // adds/s
+            cudaEventRecord(a);
+            fp32_fmnmx3_only<<<blocks, threads>>>(fo, iters, 1.5f);
+            cudaEventRecord(b); cudaEventSynchronize(b); cudaEventElapsedTime(&ms, a, b);
+            const double fm = double(blocks) * threads * double(iters) * 256 * 2 / (ms * 1e-3);   // mins/s
             const double clk = clk_khz * 1e3;                         // max SM clock
+            if (rep == (once ? 0 : 2))
+                printf("%2d warps/SM: FADD2 alone %.2f T add/s (%.1f /SM/clk), FMNMX3 alone %.2f T min/s (%.1f /SM/clk)\n",
+                       warps, fa / 1e12, fa / sms / clk, fm / 1e12, fm / sms / clk);
             if (rep == (once ? 0 : 2))
                 printf("%2d warps/SM: fp32 FADD2+FMNMX3 %.2f T add-min/s (%.1f /SM/clk at max clock), "
                        "int32 (a) %.2f T add-min/s (%.1f /SM/clk), int32 (b) xor %.2f T add-min/s (%.1f /SM/clk)\n",
