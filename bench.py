@@ -86,11 +86,39 @@ WORKLOADS = {
                              variant=0, desc="NEXT-3: generic executor, bitonic sort n=64, row-wise (Thm 2)"),
     "exec_prefix_col": dict(seed=2, algo="exec", prog="prefix", n=1024, p=2 ** 20, dtype="float32", layout=1,
                             variant=0, desc="NEXT-3: generic executor running Algorithm Prefix-sums, column-wise"),
+    # the paper's other experiment shapes (§V): n = 32K floats at p = 8K, 8-gons at
+    # p = 4M, our kernels beside the paper's naive row-/column-wise kernels (Figs. 11, 12)
+    "ps32k": dict(seed=21, algo="prefix", n=32768, p=8192, dtype="float32", layout=0, variant=0,
+                  desc="paper shape: prefix sums of n=32K floats, p=8K (P:249), row-wise, AUTO"),
+    "ps32k_col": dict(seed=21, algo="prefix", n=32768, p=8192, dtype="float32", layout=1, variant=0,
+                      desc="paper shape: prefix sums n=32K, p=8K, column-wise, AUTO"),
+    "ps32k_naive_row": dict(seed=21, algo="prefix", n=32768, p=8192, dtype="float32", layout=0, variant=5,
+                            desc="paper shape n=32K, p=8K: the paper's row-wise kernel (Fig. 11)"),
+    "ps32k_naive_col": dict(seed=21, algo="prefix", n=32768, p=8192, dtype="float32", layout=1, variant=5,
+                            desc="paper shape n=32K, p=8K: the paper's column-wise kernel (Fig. 11)"),
+    "tr8": dict(seed=23, algo="tri", n=8, p=4 * 2 ** 20, dtype="float32", layout=0, variant=0,
+                desc="paper shape: 8-gons at p=4M (P:251), fp32, row-wise, AUTO"),
+    "tr8col": dict(seed=23, algo="tri", n=8, p=4 * 2 ** 20, dtype="float32", layout=1, variant=0,
+                   desc="paper shape: 8-gons at p=4M, column-wise weights, AUTO"),
+    "tr8_umm_row": dict(seed=23, algo="tri", n=8, p=4 * 2 ** 20, dtype="float32", layout=0, variant=16,
+                        desc="paper shape 8-gons p=4M: the paper's row-wise UMM kernel (Fig. 12)"),
+    "tr8_umm_col": dict(seed=23, algo="tri", n=8, p=4 * 2 ** 20, dtype="float32", layout=1, variant=16,
+                        desc="paper shape 8-gons p=4M: the paper's column-wise UMM kernel (Fig. 12)"),
     "ps2naive_row": dict(seed=2, algo="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0, variant=5,
                          desc="the paper's row-wise kernel (thread per instance, uncoalesced)"),
 }
 EXTRAS = ["ps2col", "ps2tr", "tr_transpose", "ps1", "tr1", "tr1col", "tr1packed", "tr2", "tr2col", "tr2packed", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
-          "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col"]
+          "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col",
+          "ps32k", "ps32k_col", "ps32k_naive_row", "ps32k_naive_col", "tr8", "tr8col", "tr8_umm_row", "tr8_umm_col"]
+# The paper's own fitted GTX Titan models, in ms for p instances: context for the
+# extras of the same shape, never a target (another machine, another decade)
+PAPER_MODEL_MS = {
+    "ps1": ("row-wise 37 us + 8.09 ns * p (n=32, P:249)", lambda p: 0.037 + 8.09e-6 * p),
+    "tr8": ("row-wise 0.09 ms + 50.8 ns * p (8-gons, P:251)", lambda p: 0.09 + 50.8e-6 * p),
+    "tr8_umm_row": ("row-wise 0.09 ms + 50.8 ns * p (8-gons, P:251)", lambda p: 0.09 + 50.8e-6 * p),
+    "tr8col": ("column-wise 0.032 ms + 2.11 ns * p (8-gons, P:260)", lambda p: 0.032 + 2.11e-6 * p),
+    "tr8_umm_col": ("column-wise 0.032 ms + 2.11 ns * p (8-gons, P:260)", lambda p: 0.032 + 2.11e-6 * p),
+}
 L2_BYTES = 126 * 2 ** 20
 
 
@@ -397,6 +425,10 @@ def measure(ctx, name, steps, warmup, stream, peaks, traffic):
                            "frac": gbs / peaks["hbm_gbs"], "traffic": traffic.get(name, {}).get("dram_bytes_per_launch")}
     else:
         res["roofline"] = tri_roofline(wl, ms * steps / max(1, launches), peaks)
+    if name in PAPER_MODEL_MS:
+        what, model = PAPER_MODEL_MS[name]
+        res["paper_gtx_titan_model"] = {"ms_per_step": model(wl["p"]), "model": what,
+                                        "note": "the paper's fitted model on its GTX Titan: context, not a target"}
     return res, st
 
 
@@ -411,7 +443,7 @@ def tri_roofline(wl, per_launch_ms, peaks):
     alu = alu_peak_taddmin(peaks, wl["dtype"])
     hbm = {"bound": "hbm", "achieved": gbs, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": gbs / peaks["hbm_gbs"]}
     alu_r = {"bound": "alu", "achieved": tops, "peak": alu, "unit": "T add-min/s", "frac": tops / alu,
-             "peak_source": "measured inner mix, tools/micro/addmin_peak.cu (profiles/r01/addmin_peak.log)"}
+             "peak_source": "measured, profiles/r02/addmin_peak.json (tools/micro/addmin_peak.cu: single-pipe probes at 99 % pipe utilisation)"}
     t_hbm = algo_bytes_per_instance(wl) * p / (peaks["hbm_gbs"] * 1e9)
     t_alu = addmin_per_instance(wl) * p / (alu * 1e12)
     main, other = (hbm, alu_r) if t_hbm >= t_alu else (alu_r, hbm)
@@ -421,17 +453,20 @@ def tri_roofline(wl, per_launch_ms, peaks):
     return out
 
 
+ADDMIN_PEAK_JSON = os.path.join(ROOT, "profiles", "r02", "addmin_peak.json")
+
+
 def alu_peak_taddmin(peaks, dtype):
-    """ALU roof for the min-plus inner step, MEASURED (SURVEY §8 d: R_addmin from a
-    microbenchmark of the actual inner instruction mix): tools/micro/addmin_peak.cu
-    runs the 4x4 chunk of tri_tiled.cu from registers on all 148 SMs --
-    fp32 FADD2 + FMNMX3 68.5, int32 VIADDMNMX 61.5 add-mins per SM per clock
-    (profiles/r01/addmin_peak.log); scaled by the SM count and max clock.
-    (One add-min per lane per cycle, 128 per SM-clock, is what the unit counts
-    suggest; the measured mix reaches half of it.)"""
+    """ALU roof for the min-plus inner step, MEASURED (SURVEY §8 d): read from the
+    committed profiles/r02/addmin_peak.json (tools/micro/addmin_peak.cu on B200):
+    fp32 -- the slower of FADD2 alone (FMA pipe at 99.5 %) and FMNMX3 alone (ALU
+    pipe at 98.9 %), 121.9 add-mins per SM-clock; int32 -- the fastest measured
+    form, 71.0.  Scaled by 148 SMs and the max SM clock."""
+    with open(ADDMIN_PEAK_JSON) as fh:
+        d = json.load(fh)
+    per_sm_clk = d["fp32" if dtype == "float32" else "int32"]["roof_per_sm_clk"]
     mhz = peaks.get("sm_max_mhz", 1965.0)
-    per_sm_clk = 68.5 if dtype == "float32" else 61.5
-    return 148 * per_sm_clk * mhz * 1e6 / 1e12
+    return d["sm_count"] * per_sm_clk * mhz * 1e6 / 1e12
 
 
 def cpu_baseline(ctx, name, st, budget_s=12.0):
