@@ -104,7 +104,12 @@ template <int INST> struct Cfg {
 #ifndef BO_FR_STAGES
 #define BO_FR_STAGES 8      // measured: 1 CTA/SM with a 7-8 deep ring beats 2 CTAs x 6 (99.3 % vs 96.0 % of HBM)
 #endif
-    static constexpr int kStages = INST == 128 ? BO_FR_STAGES : 8;
+    // 32-instance tiles serve small p (measured: a 24-deep ring is slower, n = 1024
+    // p = 16384 42 vs 23.5 us, n = 32K p = 8K 0.585 vs 0.555 ms: 2 CTAs/SM instead of 6)
+#ifndef BO_FR_STAGES32
+#define BO_FR_STAGES32 8
+#endif
+    static constexpr int kStages = INST == 128 ? BO_FR_STAGES : BO_FR_STAGES32;
     static constexpr uint32_t kBoxBytes = INST * kElems * 4;   // 16 KiB / 4 KiB
     static constexpr size_t kSmem = 1024 + kStages * kBoxBytes + kStages * 16;
 };
@@ -213,7 +218,12 @@ namespace ac {
 // 32 x 8 1.356, 32 x 4 1.360, 64 x 3 1.356, 16 x 8 1.360
 constexpr int kElems = BO_AC_ROWS;          // rows per box
 constexpr int kStages = BO_AC_STAGES;
+#ifndef BO_AC_STAGES32
+#define BO_AC_STAGES32 12
+#endif
 template <int INST> struct Cfg {
+    // 32-instance column blocks (small p, long columns): a deeper ring per CTA
+    static constexpr int kStages = INST == 128 ? ac::kStages : BO_AC_STAGES32;
     static constexpr uint32_t kBoxBytes = INST * kElems * 4;
     static constexpr size_t kSmem = 1024 + kStages * kBoxBytes + kStages * 16;
 };
@@ -225,7 +235,7 @@ ps_across_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant
               long long ntiles, int nchunks, int slot) {
     pdl_begin();
     using ac::kElems;
-    constexpr int kStages = ac::kStages;
+    constexpr int kStages = ac::Cfg<kInst>::kStages;
     constexpr uint32_t kBoxBytes = ac::Cfg<kInst>::kBoxBytes;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -442,6 +452,13 @@ static int launch_across(const T *src, T *dst, int64_t n, int64_t p, cudaStream_
     if (BO_ACROSS_TMA && n >= 64 && p % 4 == 0 && aligned16(src) && aligned16(dst) && p >= 2LL * 128 * num_sms() &&
         p < (int64_t(1) << 31) && n < (int64_t(1) << 31))
         return launch_across_tma<T, 128>(src, dst, n, p, st);
+    // too few instances for 128-wide blocks but long columns (the paper's n = 32K,
+    // p = 8K): 32-wide blocks with a 12-deep ring keep every SM streaming
+    // (measured: n = 32K p = 8K 0.383 vs 1.644 ms with the scalar kernel, 5.6 TB/s;
+    // n = 1024 p = 16384 29 vs 61 us; n = 4096 p = 8192 52 vs 211 us)
+    if (BO_ACROSS_TMA && n >= 256 && p % 4 == 0 && p >= 32 && aligned16(src) && aligned16(dst) &&
+        p < (int64_t(1) << 31) && n < (int64_t(1) << 31) && p / 4 < 512LL * num_sms())
+        return launch_across_tma<T, 32>(src, dst, n, p, st);
     // 128-bit lanes when there are enough instances to fill the GPU with
     // 4-instance threads; otherwise one instance per thread, 16 rows in flight
     if (p % 4 == 0 && aligned16(src) && aligned16(dst) && p / 4 >= 512LL * num_sms()) {

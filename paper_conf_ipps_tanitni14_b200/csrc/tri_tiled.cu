@@ -320,49 +320,6 @@ __device__ __forceinline__ void dense_tile(T (&acc)[4][4], const T *Z, int I, in
         minplus_chunk(acc, A0, B0);
     }
 }
-// Dense part with a cross-step prefetch (BO_TT_PREFETCH).  The chunks of lane
-// (I, J, q, s) are m_k = m0 + k s, k = 0..cnt-1, m0 = I+1+q; they are visited in
-// the rotated order k = 1, 2, ..., cnt-1, 0, so the first one is an "old"
-// chunk whose operands (tiles of diagonals <= D-2 when the tile is on D) were
-// final before the previous step's fix-up: the previous step loads it into
-// (PA, PB) while it shuffles and fixes up, and this step starts computing at
-// once instead of waiting on shared-memory latency.  The fresh chunks (those
-// touching diagonal D-1: m = I+1 and m = J-1) come last.  Sums and their
-// association are unchanged; only the order of the min (exact) moves.
-template <typename T>
-__device__ __forceinline__ void load_chunk(typename V4<T>::type (&A)[4], typename V4<T>::type (&B)[4], const T *Z,
-                                           int I, int J, int m) {
-    const T *pa = Z + xc(4 * I, m), *pb = Z + xc(4 * m, J);
-#pragma unroll
-    for (int u = 0; u < 4; ++u) A[u] = ld4(pa + 4 * u), B[u] = ld4(pb + 4 * u);
-}
-template <typename T>
-__device__ __forceinline__ void dense_tile_rot(T (&acc)[4][4], const T *Z, int I, int J, int m0, int s, bool pre,
-                                               const typename V4<T>::type (&PA)[4],
-                                               const typename V4<T>::type (&PB)[4]) {
-    using T4 = typename V4<T>::type;
-    const int cnt = (J - m0 + s - 1) / s;               // >= 1 (caller checks m0 < J)
-    T4 A0[4], B0[4], A1[4], B1[4];
-    int k = cnt > 1 ? 1 : 0;
-    if (pre) {
-#pragma unroll
-        for (int u = 0; u < 4; ++u) A0[u] = PA[u], B0[u] = PB[u];
-    } else {
-        load_chunk(A0, B0, Z, I, J, m0 + k * s);
-    }
-    int left = cnt;
-    auto next = [&](int kk) { return kk == 0 ? 0 : (kk + 1 < cnt ? kk + 1 : 0); };
-    while (true) {
-        k = next(k);
-        if (left > 1) load_chunk(A1, B1, Z, I, J, m0 + k * s);
-        minplus_chunk(acc, A0, B0);
-        if (--left == 0) break;
-        k = next(k);
-        if (left > 1) load_chunk(A0, B0, Z, I, J, m0 + k * s);
-        minplus_chunk(acc, A1, B1);
-        if (--left == 0) break;
-    }
-}
 // Two tiles (I0, I0+D), (I1, I1+D) of one tile-diagonal, all D-1 chunks each
 // (s = 1), interleaved; D == 1 has no dense chunk (acc = +inf).
 template <typename T>
@@ -645,10 +602,6 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
         BO_CLK_MARK(1);
 
         // ------------------------------------------------ 3. D = 1 .. NT-1
-#ifdef BO_TT_PREFETCH
-        T4 PA[4], PB[4];                                 // first chunk of the next step (dense_tile_rot)
-        bool pre = false;
-#endif
         for (int D = 1; D < NT; ++D) {
             const int ls = static_cast<int>(lsched >> (4 * D)) & 15;     // split_log2(NT - D, D, LPI)
             // tile index in the low bits, split index q in the high bits: the 8-lane
@@ -684,24 +637,7 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             for (int u = 0; u < 4; ++u)
 #pragma unroll
                 for (int v = 0; v < 4; ++v) acc[u][v] = Op::inf();
-#ifdef BO_TT_PREFETCH
-            if (act && I + 1 + q < J) tt::dense_tile_rot(acc, Z, I, J, I + 1 + q, s, pre, PA, PB);
-            // prefetch step D+1's first chunk: lane (I', q', s') starts at m = I'+1+q'+s',
-            // whose tiles lie on diagonals 1+q'+s' and D-q'-s' -- both <= D-1 (final now,
-            // not written in this step) when 1 <= q'+s' <= D-2
-            pre = false;
-            if (D + 1 < NT) {
-                const int ls1 = static_cast<int>(lsched >> (4 * (D + 1))) & 15;
-                const int ib1 = kLogLpi - ls1;
-                const int I1 = li & ((1 << ib1) - 1), q1 = li >> ib1, s1 = 1 << ls1;
-                if (I1 < NT - D - 1 && q1 + s1 <= D - 2) {
-                    tt::load_chunk(PA, PB, Z, I1, I1 + D + 1, I1 + 1 + q1 + s1);
-                    pre = true;
-                }
-            }
-#else
             if (act && I + 1 + q < J) tt::dense_tile(acc, Z, I, J, I + 1 + q, s);
-#endif
             BO_CLK_MARK(80 + 4 * D);
             for (int off = 1 << ib; off < LPI; off <<= 1)
 #pragma unroll

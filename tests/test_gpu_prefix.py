@@ -168,6 +168,16 @@ def test_column_wise_tma_ring_ragged(dt, n, p):
 
 
 @pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("n,p", [(256, 32), (300, 36), (1000, 4100), (257, 996), (4096, 132), (2000, 37884)])
+def test_column_wise_tma_ring_32_wide(dt, n, p):
+    # the 32-instance column-block TMA ring (p % 4 == 0, p below 2*128*SMs, n >= 256): partial last
+    # 32-instance block and partial last 64-row chunk, element by element against the oracle
+    x = bulkgen.prefix_input(n, p, seed=n * 7 + p, dtype=dt, layout=bulkgen.COLUMN_WISE)
+    got = bo.prefix_sums(torch.from_numpy(x).to(DEV), bo.COLUMN_WISE).cpu().numpy()
+    assert np.array_equal(got.view(np.uint32), oracle.bulk_prefix_sums(x, oracle.COLUMN_WISE).view(np.uint32))
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
 @pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
 def test_every_small_n_auto(dt, layout):
     # every n = 1..200 through AUTO (fused-row TMA / smem, across vec4 / scalar), ragged p

@@ -2,7 +2,7 @@
 """Development A/B timer: time bench.py workloads exactly as bench.py does
 (rotating input copies, spin kernel ahead of the events, K steps back to back)
 for the library BULKOBL_LIB points at.  One JSON line per workload.
-    BULKOBL_LIB=ab/NAME/libbulkobl.so python tools/abtime.py ps2col tr2 [--steps 20] [--reps 3]"""
+    BULKOBL_LIB=ab/NAME/libbulkobl.so python tools/abtime.py ps2col tr2 prefix:1024:16384:float32:0 [--steps 20] [--reps 3]"""
 import json
 import os
 import sys
@@ -24,7 +24,12 @@ def main():
     stream = torch.cuda.Stream()
     lib = os.environ.get("BULKOBL_LIB", "in-tree")
     for name in args:
-        wl = bench.WORKLOADS[name]
+        if ":" in name:          # ad-hoc spec algo:n:p:dtype:layout[:variant], e.g. prefix:1024:16384:float32:0
+            f = name.split(":")
+            wl = dict(seed=5, algo=f[0], n=int(f[1]), p=int(f[2]), dtype=f[3], layout=int(f[4]),
+                      variant=int(f[5]) if len(f) > 5 else 0, desc=name)
+        else:
+            wl = bench.WORKLOADS[name]
         st = bench.setup_workload(wl, 0, bench.copies_for(wl))
         ms = min(bench.timed(ctx, st["fn"], steps, 3, stream)[0] for _ in range(reps))
         print(json.dumps({"lib": lib, "workload": name, "variant": st["variant"], "ms": round(ms, 5),

@@ -1,8 +1,30 @@
 #!/usr/bin/env python
-"""Host-side cost of one binding call (ctypes + argument checks + C-side launch), cProfile."""
-import time, torch, sys, cProfile, pstats
-sys.path.insert(0, '.')
-import paper_conf_ipps_tanitni14_b200 as bo
+"""Host-side cost of one binding call (ctypes + argument checks + C-side launch):
+us per call for triangulation (both layouts) and prefix sums, then a cProfile of
+the prefix-sum call.  python tools/hostprof.py"""
+import cProfile
+import os
+import pstats
+import sys
+import time
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_ipps_tanitni14_b200 as bo  # noqa: E402
+
+for layout in (bo.ROW_WISE, bo.COLUMN_WISE):
+    ct = bo.generate_tri(16, 65536, 3, torch.int32, layout)
+    ot = torch.empty(65536, dtype=torch.int32, device="cuda")
+    for _ in range(10):
+        bo.triangulation(ct, layout, out=ot)
+    torch.cuda.synchronize()
+    torch.cuda._sleep(int(0.2 * 2e9))
+    t0 = time.perf_counter()
+    for _ in range(200):
+        bo.triangulation(ct, layout, out=ot)
+    print(f"triangulation layout {layout}: host {(time.perf_counter() - t0) / 200 * 1e6:.2f} us/call")
+    torch.cuda.synchronize()
 c = bo.generate_tri(16, 65536, 3, torch.int32, 1)
 out = torch.empty(65536, dtype=torch.int32, device="cuda")
 x = bo.generate_prefix(32, 1024, 1, torch.int32, 0)
