@@ -54,13 +54,16 @@ __host__ __device__ __forceinline__ long long c_index(int layout, long long h, l
 }
 
 // -------------------------------------------------------------- THREAD_REG
+#ifndef BO_REG_THREADS
+#define BO_REG_THREADS 256   // measured TR-1 column-wise: 256 7.11 us, 128 7.32, 64 7.22, 32 7.22
+#endif
 template <typename T, int N, int LAYOUT>   // layout a template parameter: the 105+ weight
-__global__ void __launch_bounds__(128)      // loads must be branch-free so they issue early
+__global__ void __launch_bounds__(BO_REG_THREADS)      // loads must be branch-free so they issue early
 tri_thread_reg(const T *__restrict__ c, T *__restrict__ out, long long p) {
     pdl_begin();
     constexpr int layout = LAYOUT;
     using Op = MinPlus<T>;
-    const long long h = blockIdx.x * 128LL + threadIdx.x;
+    const long long h = static_cast<long long>(blockIdx.x) * BO_REG_THREADS + threadIdx.x;
     if (h >= p) return;
     T M[N][N];                         // 1-based M[i][j], i <= j; all indices compile-time
 #pragma unroll
@@ -414,14 +417,14 @@ static int launch_reg_n(const void *c, void *out, int64_t p, int layout, cudaStr
         if (layout == BO_ROW_WISE && (N * N) % 4 == 0) return launch_reg_tma<T, N, BO_ROW_WISE>(c, out, p, st);
         // column-wise c is already coalesced for thread-per-instance: direct loads win (measured 14.5 vs 19.3 us)
     }
-    const unsigned grid = static_cast<unsigned>((p + 127) / 128);
+    const unsigned grid = static_cast<unsigned>((p + BO_REG_THREADS - 1) / BO_REG_THREADS);
     const T *cc = static_cast<const T *>(c);
     T *oo = static_cast<T *>(out);
     switch (layout) {
-        case BO_ROW_WISE: launch(tri_thread_reg<T, N, BO_ROW_WISE>, grid, 128, 0, st, cc, oo, p); break;
-        case BO_COLUMN_WISE: launch(tri_thread_reg<T, N, BO_COLUMN_WISE>, grid, 128, 0, st, cc, oo, p); break;
-        case BO_PACKED_ROW: launch(tri_thread_reg<T, N, BO_PACKED_ROW>, grid, 128, 0, st, cc, oo, p); break;
-        default: launch(tri_thread_reg<T, N, BO_PACKED_COLUMN>, grid, 128, 0, st, cc, oo, p); break;
+        case BO_ROW_WISE: launch(tri_thread_reg<T, N, BO_ROW_WISE>, grid, BO_REG_THREADS, 0, st, cc, oo, p); break;
+        case BO_COLUMN_WISE: launch(tri_thread_reg<T, N, BO_COLUMN_WISE>, grid, BO_REG_THREADS, 0, st, cc, oo, p); break;
+        case BO_PACKED_ROW: launch(tri_thread_reg<T, N, BO_PACKED_ROW>, grid, BO_REG_THREADS, 0, st, cc, oo, p); break;
+        default: launch(tri_thread_reg<T, N, BO_PACKED_COLUMN>, grid, BO_REG_THREADS, 0, st, cc, oo, p); break;
     }
     return after_launch("tri_thread_reg");
 }
