@@ -92,6 +92,14 @@ tri_thread_reg(const T *__restrict__ c, T *__restrict__ out, long long p) {
 // flight while W compute.  (Measured: p = 2^20 156 us with W = 2, S = 4 against
 // 161 us with one-warp CTAs; p = 65536 is DRAM-bound either way, 14.4 us.)  Only elements up to the last one Algorithm OPT
 // reads are fetched.
+// Box width in elements of the row-wise TMA batches: 32 (128-byte rows, 128B
+// swizzle), or 16 (64-byte rows, 64B swizzle) where that fetches fewer of the
+// elements past the last one Algorithm OPT reads -- n = 8: 48 of 64 elements
+// (192 instead of 256 bytes per instance), n = 10: 80 of 100 (320 instead of 384).
+__host__ __device__ constexpr int reg_tma_box_width(int N, int layout) {
+    return layout == BO_ROW_WISE && (N == 8 || N == 10) ? 16 : 32;
+}
+
 template <typename T, int N, int LAYOUT, int S, int W>
 __global__ void __launch_bounds__(32 * W)
 tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out, long long p, long long nbatch) {
@@ -99,8 +107,10 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
     using Op = MinPlus<T>;
     constexpr int NE = LAYOUT == BO_PACKED_ROW ? (N - 1) * (N - 2) / 2   // packed: every weight is read
                                                : (N - 3) * N + N;        // c[N-3][N-1] is the last one read
-    constexpr int NB = (NE + 31) / 32;
-    constexpr uint32_t kBatchBytes = NB * 4096;
+    constexpr int BW = reg_tma_box_width(N, LAYOUT);   // elements per box row (32, or 16 with 64B swizzle)
+    constexpr int NB = (NE + BW - 1) / BW;
+    constexpr uint32_t kBoxBytes = 32u * BW * 4u;
+    constexpr uint32_t kBatchBytes = NB * kBoxBytes;
     // slot i % S of batch i is then always one of warp i % W's own slots: a warp
     // can never wait on (or refill) a slot whose previous batch another warp
     // still holds, so one full barrier per slot and its phase parity suffice
@@ -117,8 +127,8 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
         mbar_arrive_expect_tx(&bar[sl], kBatchBytes);
 #pragma unroll
         for (int k = 0; k < NB; ++k) {
-            if (LAYOUT != BO_COLUMN_WISE) tma_load_2d(dst + k * 4096, &cmap, k * 32, static_cast<int>(b * 32), &bar[sl]);
-            else tma_load_2d(dst + k * 4096, &cmap, static_cast<int>(b * 32), k * 32, &bar[sl]);
+            if (LAYOUT != BO_COLUMN_WISE) tma_load_2d(dst + k * kBoxBytes, &cmap, k * BW, static_cast<int>(b * 32), &bar[sl]);
+            else tma_load_2d(dst + k * kBoxBytes, &cmap, static_cast<int>(b * 32), k * 32, &bar[sl]);
         }
     };
     if (threadIdx.x == 0) {
@@ -141,9 +151,13 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
                 const int a = e / N, b = e % N;
                 e = a * (N - 2) - a * (a - 1) / 2 + (b - a - 2);
             }
-            const uint8_t *box = cur + (e >> 5) * 4096;
+            const uint8_t *box = cur + (e / BW) * kBoxBytes;
             if (LAYOUT != BO_COLUMN_WISE) {
-                const uint4 v = *reinterpret_cast<const uint4 *>(box + swz128(t, (e & 31) >> 2));
+                // 128B swizzle: chunk ^ (row % 8) in 128-byte rows; 64B swizzle: chunk ^ ((row / 2) % 4)
+                // in 64-byte rows -- either way the 8 lanes of a phase hit 8 distinct 16-byte slots
+                const int ch = (e % BW) >> 2;
+                const uint32_t off = BW == 32 ? swz128(t, ch) : t * 64u + ((ch ^ ((t >> 1) & 3)) << 4);
+                const uint4 v = *reinterpret_cast<const uint4 *>(box + off);
                 const uint32_t w = (e & 3) == 0 ? v.x : (e & 3) == 1 ? v.y : (e & 3) == 2 ? v.z : v.w;
                 return *reinterpret_cast<const T *>(&w);
             }
@@ -363,7 +377,7 @@ size_t tri_workspace(int64_t n, int64_t p, int variant) {
 }
 
 // ring geometry of the TMA-fed THREAD_REG kernel: W warps per CTA (one CTA per
-// SM), S batch slots of NB*4 KB
+// SM), S batch slots of NB boxes of [32 instances x BW elements]
 #ifndef BO_REG_TMA_STAGES
 #define BO_REG_TMA_STAGES 4
 #endif
@@ -374,11 +388,13 @@ template <typename T, int N, int LAYOUT>
 static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) {
     constexpr int S = BO_REG_TMA_STAGES, W = BO_REG_TMA_WARPS;
     constexpr int NE = (N - 3) * N + N;
-    constexpr int NB = (NE + 31) / 32;
-    constexpr size_t smem = 1024 + S * NB * 4096 + 8 * S;
+    constexpr int BW = reg_tma_box_width(N, LAYOUT);
+    constexpr int NB = (NE + BW - 1) / BW;
+    constexpr size_t smem = 1024 + S * NB * (32 * BW * 4) + 8 * S;
     CUtensorMap map;
     constexpr int K = (N - 1) * (N - 2) / 2;
-    const bool ok = LAYOUT == BO_ROW_WISE     ? make_tmap_2d(&map, c, p, N * N, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
+    const bool ok = LAYOUT == BO_ROW_WISE     ? make_tmap_2d(&map, c, p, N * N, 32, BW,
+                                                             BW == 16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B)
                     : LAYOUT == BO_PACKED_ROW ? make_tmap_2d(&map, c, p, K, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
                                               : make_tmap_2d(&map, c, N * N, p, 32, 32, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (!ok) return fail(BO_ECUDA, "triangulation THREAD_REG: cuTensorMapEncodeTiled failed");

@@ -86,6 +86,20 @@ def test_argument_validation_without_gpu(L):
     assert L.bulk_transpose(p, p, 0, 4, 4, None) == 0
 
 
+def test_workspace_overlap_and_alignment_rejected_without_gpu(L):
+    # a prefix workspace may share no byte with src or dst; TILED_GLOBAL's workspace
+    # must be 16-byte aligned (both checked before any CUDA call)
+    src, dst = ctypes.c_void_p(1 << 20), ctypes.c_void_p(2 << 20)
+    n, p = 4, 4                                                   # 64 bytes each
+    need = n * p * 4
+    for ws in ((2 << 20) + 16, (2 << 20) - 16, (1 << 20) + 60, (1 << 20) - 60):
+        assert L.bulk_prefix_sums(src, dst, n, p, 0, 0, bo.PS_TRANSPOSED, ctypes.c_void_p(ws), need, None) == -1
+        assert b"workspace overlaps" in L.bulk_last_error()
+    assert L.bulk_triangulation(src, dst, 100, 8, 1, 0, bo.TRI_TILED_GLOBAL, ctypes.c_void_p((3 << 20) + 4),
+                                1 << 30, None) == -1
+    assert b"16-byte aligned" in L.bulk_last_error()
+
+
 def test_workspace_and_variant_queries(L):
     assert bo.triangulation_workspace(64, 1000, bo.F32, bo.COLUMN_WISE, bo.TRI_UMM_GLOBAL) == 63 * 63 * 1000 * 4
     assert bo.triangulation_workspace(64, 1000, bo.F32, bo.COLUMN_WISE, bo.TRI_SMEM_WARP) == 0

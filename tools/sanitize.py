@@ -11,7 +11,7 @@ import torch  # noqa: E402
 import paper_conf_ipps_tanitni14_b200 as bo  # noqa: E402
 
 for layout in (bo.ROW_WISE, bo.COLUMN_WISE):
-    for n, p in ((64, 300), (33, 129), (1024, 260)):
+    for n, p in ((64, 300), (33, 129), (1024, 260), (300, 100)):   # (300, 100) column-wise: the 32-wide TMA ring
         x = bo.generate_prefix(n, p, 1, torch.float32, layout)
         vs = [bo.AUTO, bo.PS_NAIVE] + ([bo.PS_FUSED_ROW, bo.PS_WARPSCAN, bo.PS_TRANSPOSED] if layout == 0 else
                                        [bo.PS_ACROSS])
