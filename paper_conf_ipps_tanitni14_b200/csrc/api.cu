@@ -115,7 +115,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 }
 
 bool make_tmap_2d(CUtensorMap *map, const void *base, uint64_t rows, uint64_t cols, uint32_t box_rows,
-                  uint32_t box_cols, CUtensorMapSwizzle swz) {
+                  uint32_t box_cols, CUtensorMapSwizzle swz, CUtensorMapL2promotion l2) {
     // The encoded map depends only on these arguments, so a repeated call on the
     // same buffer and shape reuses it: encoding costs several microseconds of
     // host time, more than a small config's kernel (thread-local, 16 entries).
@@ -123,7 +123,7 @@ bool make_tmap_2d(CUtensorMap *map, const void *base, uint64_t rows, uint64_t co
         const void *base;
         uint64_t rows, cols;
         uint32_t box_rows, box_cols;
-        int swz;
+        int swz, l2;
         CUtensorMap map;
     };
     static thread_local Entry memo[16];
@@ -131,7 +131,7 @@ bool make_tmap_2d(CUtensorMap *map, const void *base, uint64_t rows, uint64_t co
     for (int i = 0; i < filled; ++i) {
         const Entry &e = memo[i];
         if (e.base == base && e.rows == rows && e.cols == cols && e.box_rows == box_rows && e.box_cols == box_cols &&
-            e.swz == static_cast<int>(swz)) {
+            e.swz == static_cast<int>(swz) && e.l2 == static_cast<int>(l2)) {
             *map = e.map;
             return true;
         }
@@ -143,10 +143,10 @@ bool make_tmap_2d(CUtensorMap *map, const void *base, uint64_t rows, uint64_t co
     cuuint32_t box[2] = {box_cols, box_rows};
     cuuint32_t es[2] = {1, 1};
     CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void *>(base), dims, strides, box, es,
-                    CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, swz, l2,
                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return false;
-    memo[next] = Entry{base, rows, cols, box_rows, box_cols, static_cast<int>(swz), *map};
+    memo[next] = Entry{base, rows, cols, box_rows, box_cols, static_cast<int>(swz), static_cast<int>(l2), *map};
     next = (next + 1) % 16;
     filled = filled < 16 ? filled + 1 : 16;
     return true;

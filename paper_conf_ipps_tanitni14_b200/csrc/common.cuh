@@ -80,7 +80,8 @@ inline int num_sms() {
 // 2-D tensor map over a row-major [rows][cols] array of 4-byte elements.
 // box = {box_cols, box_rows}; swizzle 128B requires box_cols*4 <= 128.
 bool make_tmap_2d(CUtensorMap *map, const void *base, uint64_t rows, uint64_t cols,
-                  uint32_t box_rows, uint32_t box_cols, CUtensorMapSwizzle swz);
+                  uint32_t box_rows, uint32_t box_cols, CUtensorMapSwizzle swz,
+                  CUtensorMapL2promotion l2 = CU_TENSOR_MAP_L2_PROMOTION_L2_256B);
 
 inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 

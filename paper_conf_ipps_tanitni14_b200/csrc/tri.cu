@@ -94,10 +94,11 @@ tri_thread_reg(const T *__restrict__ c, T *__restrict__ out, long long p) {
 // reads are fetched.
 // Box width in elements of the row-wise TMA batches: 32 (128-byte rows, 128B
 // swizzle), or 16 (64-byte rows, 64B swizzle) where that fetches fewer of the
-// elements past the last one Algorithm OPT reads -- n = 8: 48 of 64 elements
-// (192 instead of 256 bytes per instance), n = 10: 80 of 100 (320 instead of 384).
+// elements past the last one Algorithm OPT reads: n = 8, 48 of 64 elements
+// (192 instead of 256 bytes per instance; with L2 promotion to 64 B, 8-gons at
+// p = 4M 159 -> 131 us).  n = 10 (80 of 100) measured slower (76 vs 68 us at p = 2^20).
 __host__ __device__ constexpr int reg_tma_box_width(int N, int layout) {
-    return layout == BO_ROW_WISE && (N == 8 || N == 10) ? 16 : 32;
+    return layout == BO_ROW_WISE && N == 8 ? 16 : 32;
 }
 
 template <typename T, int N, int LAYOUT, int S, int W>
@@ -393,8 +394,21 @@ static int launch_reg_tma(const void *c, void *out, int64_t p, cudaStream_t st) 
     constexpr size_t smem = 1024 + S * NB * (32 * BW * 4) + 8 * S;
     CUtensorMap map;
     constexpr int K = (N - 1) * (N - 2) / 2;
-    const bool ok = LAYOUT == BO_ROW_WISE     ? make_tmap_2d(&map, c, p, N * N, 32, BW,
-                                                             BW == 16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B)
+    // Boxes that stop short of an instance's last bytes save DRAM traffic only if L2
+    // does not promote the requests back to whole 256-byte lines.  Measured: n = 8
+    // (16-element boxes) p = 4M 131 us with 64B promotion, 159 us with 256B, 161 us
+    // with none; n = 16 (32-element boxes, 896 of 1024 bytes) p = 65536 10.9-11.0 us
+    // with 64B / 128B / none against 12.0 us with 256B (p = 2^20: 138 vs 154 us).
+#ifndef BO_REG_BW16_L2
+#define BO_REG_BW16_L2 CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+#endif
+#ifndef BO_REG_L2
+#define BO_REG_L2 CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+#endif
+    const bool ok = LAYOUT == BO_ROW_WISE     ? (BW == 16 ? make_tmap_2d(&map, c, p, N * N, 32, BW, CU_TENSOR_MAP_SWIZZLE_64B,
+                                                                         BO_REG_BW16_L2)
+                                                          : make_tmap_2d(&map, c, p, N * N, 32, BW, CU_TENSOR_MAP_SWIZZLE_128B,
+                                                                         BO_REG_L2))
                     : LAYOUT == BO_PACKED_ROW ? make_tmap_2d(&map, c, p, K, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)
                                               : make_tmap_2d(&map, c, N * N, p, 32, 32, CU_TENSOR_MAP_SWIZZLE_NONE);
     if (!ok) return fail(BO_ECUDA, "triangulation THREAD_REG: cuTensorMapEncodeTiled failed");

@@ -11,11 +11,11 @@
 // c[a][b] and X[a][b] share coordinates, so c is preloaded into the table.
 //
 // Shared-memory table: the UPPER triangle only, stored by 4-wide column
-// chunks ("chunk-columns"): chunk-column m holds rows 0..4m+2 of columns
-// 4m..4m+3, so element X[a][b] lives at chunk colbase(b/4) + a, word b%4, with
-// colbase(m) = 2m^2 + m (heights 4m+3 are odd, which spreads the quarter-warp's
-// chunks over all 8 bank groups; row 4m+2 is all zero, see colbase).  8.25 KB
-// per instance at n = 64 instead of a 16 KB square.
+// chunks ("chunk-columns"): chunk-column m holds rows 0..4m+3 (+1 pad row) of
+// columns 4m..4m+3, so element X[a][b] lives at chunk colbase(b/4) + a, word
+// b%4, with colbase(m) = 2m^2 + 3m (heights 4m+5 are odd, which spreads the
+// quarter-warp's chunks over all 8 bank groups).  8.75 KB per instance at
+// n = 64 instead of a 16 KB square, so twice as many instances per SM.
 // Before a cell is computed it holds c[a][b] (preloaded with cp.async).
 // For a tile (I,J), I < J (rows 4I..4I+3, cols 4J..4J+3) the k range splits
 //   k in [4I+4, 4J-1]  -> dense min-plus product over chunk-columns m = I+1..J-1:
@@ -85,20 +85,10 @@ template <typename T> struct V4;
 template <> struct V4<float> { using type = float4; };
 template <> struct V4<int32_t> { using type = int4; };
 
-// chunk-column m starts at chunk colbase(m); element (a, b) at word xoff(a, b).
-// CB = 1 (shared-memory kernels): chunk-column m has height 4m+3 -- the rows
-// 0..4m+1 that hold cells with b > a+1, then row 4m+2, which is never written
-// and stays 0: it doubles as the polygon edge X[4m+2][4m+3] = 0 and as the
-// pad that keeps heights odd.  Row 4m+3 of the diagonal tile (all lower
-// triangle) is not stored.  8.25 KB per instance at n = 64, so 13 warps (26
-// instances) fit one SM.  CB = 3 (TILED_GLOBAL): height 4m+5, the whole
-// diagonal tile plus a pad row.
-template <int CB = 1>
-__host__ __device__ __forceinline__ constexpr int colbase(int m) { return 2 * m * m + CB * m; }
-template <int CB = 1>
-__device__ __forceinline__ int xc(int a, int m) { return 4 * (colbase<CB>(m) + a); }   // chunk (row a, col-chunk m)
-template <int CB = 1>
-__device__ __forceinline__ int xoff(int a, int b) { return xc<CB>(a, b >> 2) + (b & 3); }
+// chunk-column m starts at chunk colbase(m); element (a, b) at word xoff(a, b)
+__host__ __device__ __forceinline__ constexpr int colbase(int m) { return 2 * m * m + 3 * m; }
+__device__ __forceinline__ int xc(int a, int m) { return 4 * (colbase(m) + a); }   // chunk (row a, col-chunk m)
+__device__ __forceinline__ int xoff(int a, int b) { return xc(a, b >> 2) + (b & 3); }
 
 template <typename T>
 __device__ __forceinline__ typename V4<T>::type ld4(const T *p) {
@@ -127,32 +117,6 @@ __device__ __forceinline__ float comp(const float4 &v, int i) { return i == 0 ? 
 __device__ __forceinline__ int comp(const int4 &v, int i) { return i == 0 ? v.x : i == 1 ? v.y : i == 2 ? v.z : v.w; }
 
 __device__ __forceinline__ void minplus_chunk(float (&acc)[4][4], const float4 (&A)[4], const float4 (&B)[4]) {
-#ifdef BO_TT_MPGROUP
-    // all 32 FADD2 of a row pair first, then the FMNMX3s (more independent work between producer and consumer)
-#pragma unroll
-    for (int u0 = 0; u0 < 4; u0 += 2) {
-        float2 sm[2][4][2];   // [u - u0][w][v pair]
-#pragma unroll
-        for (int du = 0; du < 2; ++du)
-#pragma unroll
-            for (int w = 0; w < 4; ++w) {
-                const float a = comp(A[u0 + du], w);
-                sm[du][w][0] = __fadd2_rn(make_float2(a, a), make_float2(comp(B[w], 0), comp(B[w], 1)));
-                sm[du][w][1] = __fadd2_rn(make_float2(a, a), make_float2(comp(B[w], 2), comp(B[w], 3)));
-            }
-#pragma unroll
-        for (int du = 0; du < 2; ++du)
-#pragma unroll
-            for (int vp = 0; vp < 2; ++vp) {
-                float &x0 = acc[u0 + du][2 * vp], &x1 = acc[u0 + du][2 * vp + 1];
-                x0 = fminf(fminf(x0, sm[du][0][vp].x), sm[du][1][vp].x);
-                x1 = fminf(fminf(x1, sm[du][0][vp].y), sm[du][1][vp].y);
-                x0 = fminf(fminf(x0, sm[du][2][vp].x), sm[du][3][vp].x);
-                x1 = fminf(fminf(x1, sm[du][2][vp].y), sm[du][3][vp].y);
-            }
-    }
-    return;
-#endif
 #pragma unroll
     for (int u = 0; u < 4; ++u)
 #pragma unroll
@@ -289,7 +253,7 @@ __device__ __forceinline__ void dense_tile(T (&acc)[4][4], const T *Z, int I, in
     T4 A0[4], B0[4], A1[4], B1[4];
 #pragma unroll
     for (int u = 0; u < 4; ++u) A0[u] = ld4(pa + 4 * u), B0[u] = ld4(pb + 4 * u);
-    pa += 4 * (4 * m * s + 2 * s * s + s);           // colbase(m+s) - colbase(m) chunks
+    pa += 4 * (4 * m * s + 2 * s * s + 3 * s);       // colbase(m+s) - colbase(m) chunks
     pb += db;
     m += s;
     bool more = m < J;
@@ -299,7 +263,7 @@ __device__ __forceinline__ void dense_tile(T (&acc)[4][4], const T *Z, int I, in
     }
     minplus_chunk(acc, A0, B0);
     while (more) {
-        pa += 4 * (4 * m * s + 2 * s * s + s);
+        pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
         pb += db;
         m += s;
         more = m < J;
@@ -309,7 +273,7 @@ __device__ __forceinline__ void dense_tile(T (&acc)[4][4], const T *Z, int I, in
         }
         minplus_chunk(acc, A1, B1);
         if (!more) break;
-        pa += 4 * (4 * m * s + 2 * s * s + s);
+        pa += 4 * (4 * m * s + 2 * s * s + 3 * s);
         pb += db;
         m += s;
         more = m < J;
@@ -343,7 +307,7 @@ __device__ __forceinline__ void dense_tile2(T (&acc0)[4][4], T (&acc1)[4][4], co
     minplus_first(acc0, A0, B0);
     minplus_first(acc1, A1, B1);
     for (int k = 2; k < D; ++k) {
-        pa0 += 4 * (4 * m0 + 3), pa1 += 4 * (4 * m1 + 3);       // colbase(m+1) - colbase(m) = 4m + 3 chunks
+        pa0 += 4 * (4 * m0 + 5), pa1 += 4 * (4 * m1 + 5);       // colbase(m+1) - colbase(m) = 4m + 5 chunks
         pb0 += 16, pb1 += 16;
         ++m0, ++m1;
 #pragma unroll
@@ -373,19 +337,12 @@ __device__ __forceinline__ void load_fix_operands(const T *Z, int I, int J, cons
     // A[u][w] = X[4I+u][4I+w] (w > u; registers), Bd[w][v] = X[4J+w][4J+v] (v > w),
     // C[u][v] = c[4I+u][4J+v] (still in the tile's own upper cells)
     diag_upper(A, d);
-    // (the diagonal tile's rows 2..3 are not stored: Bd[2][3] = X[4J+2][4J+3] is
-    // the polygon edge 0, the rest lower triangle; fixup<float> reads rows 0..1)
     const T *tb = Z + xc(4 * J, J), *tc = Z + xc(4 * I, J);
 #pragma unroll
     for (int r = 0; r < 4; ++r) {
-        const T4 w = ld4(tc + 4 * r);
+        const T4 y = ld4(tb + 4 * r), w = ld4(tc + 4 * r);
+        Bd[r][0] = y.x; Bd[r][1] = y.y; Bd[r][2] = y.z; Bd[r][3] = y.w;
         C[r][0] = w.x; C[r][1] = w.y; C[r][2] = w.z; C[r][3] = w.w;
-        if (r < 2) {
-            const T4 y = ld4(tb + 4 * r);
-            Bd[r][0] = y.x; Bd[r][1] = y.y; Bd[r][2] = y.z; Bd[r][3] = y.w;
-        } else {
-            Bd[r][0] = Bd[r][1] = Bd[r][2] = Bd[r][3] = T(0);
-        }
     }
 }
 // fix-up of tile (I, J = I + D) and store; X[4I+3][4I+4] is an edge of the
@@ -441,8 +398,8 @@ static uint64_t split_schedule(int NT, int lpi) {
 // Four instances per warp (LPI = 8) sit on lanes = slot mod 4 with tables
 // 8 words (mod 32) apart, the same idea one level down.
 __host__ __device__ constexpr int table_stride(int NT, int ipw) {
-    return ipw > 1 ? 4 * tt::colbase(NT) + ((32 / ipw - 4 * tt::colbase(NT)) % 32 + 32) % 32
-                   : 4 * tt::colbase(NT);
+    return ipw > 1 ? 4 * (2 * NT * NT + 3 * NT) + ((32 / ipw - 4 * (2 * NT * NT + 3 * NT)) % 32 + 32) % 32
+                   : 4 * (2 * NT * NT + 3 * NT);
 }
 
 // Step 1 of an instance: c -> upper table.  Only the weights Algorithm OPT
@@ -523,26 +480,8 @@ __device__ __forceinline__ void preload_table(T *Z, const T *__restrict__ c, lon
     }
 }
 
-// CTAs of up to kMaxWarps(LPI) warps.  (At n = 64 with 16 lanes per instance
-// one 13-warp CTA would hold 26 tables (214 KB) where 1-warp CTAs fit 24, each
-// CTA reserving 1 KB; measured slower, 0.432 vs 0.383 ms: ptxas schedules the
-// kernel into 115-125 registers under a 416-thread bound, against 148 under
-// (128, 1).  -DBO_TT_MAXW=13 builds it.)
-#ifndef BO_TT_MAXW
-#define BO_TT_MAXW 4
-#endif
-template <int LPI> constexpr int kMaxWarps = LPI == 16 ? BO_TT_MAXW : 4;
 template <typename T, int LPI, bool CHORDS>
-#if defined(BO_TT_MAXNREG)
-__global__ void __maxnreg__(BO_TT_MAXNREG)
-#elif defined(BO_TT_NOMINB)
-__global__ void __launch_bounds__(32 * kMaxWarps<LPI>)
-#else
-#ifndef BO_TT_MINB
-#define BO_TT_MINB 1
-#endif
-__global__ void __launch_bounds__(32 * kMaxWarps<LPI>, BO_TT_MINB)
-#endif
+__global__ void __launch_bounds__(128, 1)
 tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restrict__ chords, int n, long long p,
                  int layout, int NT, int c_vec, uint64_t lsched) {
     pdl_begin();
@@ -576,7 +515,9 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
         long long clk_ = clock64();
 #endif
         // ------------------------------------------------ 1. c -> upper table
+#ifndef BO_TT_NOPRELOAD
         preload_table<T, LPI>(Z, c, h, live, n, p, layout, NT, c_vec, li);
+#endif   // (-DBO_TT_NOPRELOAD: timing experiment only -- results are wrong)
         __syncwarp();
         BO_CLK_MARK(0);
 
@@ -594,7 +535,9 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             const T t13 = Op::add(Op::add(z, z), c1.w);
             const T t03 = Op::add(Op::min(Op::add(z, t13), Op::add(t02, z)), c0.w);
             tt::st4(r0, z, z, t02, t03);                 // below-diagonal words are unused
-            tt::st4(r0 + 4, z, z, z, t13);               // (row 2 is the zero row, row 3 not stored)
+            tt::st4(r0 + 4, z, z, z, t13);
+            tt::st4(r0 + 8, z, z, z, z);
+            tt::st4(r0 + 12, z, z, z, z);
             T(&dg)[3] = k == 0 ? dg0 : dg1;
             dg[0] = t02; dg[1] = t03; dg[2] = t13;
         }
@@ -734,28 +677,21 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
     const int NT = static_cast<int>((n + 3) / 4);
     constexpr int IPW = 32 / LPI;
     const size_t per_inst = static_cast<size_t>(table_stride(NT, IPW)) * sizeof(T);
-    const void *fn = reinterpret_cast<const void *>(&tri_tiled_kernel<T, LPI, CHORDS>);
-    const bool attr = ensure_dyn_smem(fn, 227 * 1024);
-    if (!attr) return fail(BO_ECUDA, "tiled: cannot set dynamic smem");
-    // warps per CTA: the W in 1..kMaxWarps that keeps the most warps resident
-    // per SM (shared memory and registers decide; occupancy query per W); ties
-    // go to the smaller W.  When p cannot fill every SM's resident warps once,
-    // spread instead: 1-warp CTAs (4 for column-wise weights, whose CTA's 8+
-    // consecutive instances share whole sectors).
-    int W = 1, best = 0, best_per_sm = 1;
-    for (int w = 1; w <= kMaxWarps<LPI>; ++w) {
-        const size_t sm_bytes = static_cast<size_t>(w) * IPW * per_inst;
-        if (sm_bytes > 227 * 1024) break;
-        const int per_sm = max_blocks_per_sm(fn, w * 32, sm_bytes);
-        if (per_sm * w > best || (layout == BO_COLUMN_WISE && w == 4 && per_sm * w == best))
-            best = per_sm * w, W = w, best_per_sm = per_sm;
-    }
-    if ((p + IPW - 1) / IPW < static_cast<long long>(best) * num_sms()) {
-        W = layout == BO_COLUMN_WISE ? 4 : 1;
-        best_per_sm = max_blocks_per_sm(fn, W * 32, static_cast<size_t>(W) * IPW * per_inst);
+    // warps per CTA: the W in 1..4 that keeps the most warps resident per SM
+    // (shared memory is the limit: 227 KB, 1 KB reserved per CTA)
+    int W = 1, best = 0;
+    for (int w = 1; w <= 4; ++w) {
+        const size_t per_cta = w * IPW * per_inst + 1024;
+        const int resident = static_cast<int>((227 * 1024) / per_cta) * w;
+        // column-wise weights: prefer 4 warps (8+ consecutive instances = whole sectors)
+        if (resident > best || (layout == BO_COLUMN_WISE && resident == best)) best = resident, W = w;
     }
     const size_t smem = W * IPW * per_inst;
-    const int per_sm = std::max(best_per_sm, 1);
+    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_tiled_kernel<T, LPI, CHORDS>), 227 * 1024);
+    if (!attr) return fail(BO_ECUDA, "tiled: cannot set dynamic smem");
+    int per_sm = 1;
+    per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&tri_tiled_kernel<T, LPI, CHORDS>), W * 32, smem);
+    per_sm = std::max(per_sm, 1);
     const long long per_cta = static_cast<long long>(W) * IPW;
     const long long blocks = std::min<long long>((p + per_cta - 1) / per_cta,
                                                  static_cast<long long>(per_sm) * num_sms());
@@ -806,7 +742,7 @@ tri_tiled_global_kernel(const T *__restrict__ c, T *__restrict__ out, T *ws, int
     using Op = tt::Ops<T>;
     using T4 = typename tt::V4<T>::type;
     using tt::xc;
-    const long long words = 4LL * tt::colbase<3>(NT);
+    const long long words = 4LL * tt::colbase(NT);
     T *Z = ws + static_cast<long long>(blockIdx.x) * words;
     const int tid = threadIdx.x, nthr = blockDim.x;
     const long long nn = static_cast<long long>(n) * n;
@@ -818,16 +754,16 @@ tri_tiled_global_kernel(const T *__restrict__ c, T *__restrict__ out, T *ws, int
             const T4 *src = reinterpret_cast<const T4 *>(c + h * nn);
             for (int idx = tid; idx < (n - 2) * NT; idx += nthr) {
                 const int a = idx / NT, m = idx - a * NT;
-                if (m >= ((a + 2) >> 2)) *reinterpret_cast<T4 *>(Z + xc<3>(a, m)) = __ldg(src + static_cast<long long>(a) * (n / 4) + m);
+                if (m >= ((a + 2) >> 2)) *reinterpret_cast<T4 *>(Z + xc(a, m)) = __ldg(src + static_cast<long long>(a) * (n / 4) + m);
             }
         } else {
             for (int a = 0; a < n - 2; ++a)
-                for (int b = a + 2 + tid; b < n; b += nthr) Z[tt::xoff<3>(a, b)] = __ldg(c + tri_c_index(layout, h, n, p, a, b));
+                for (int b = a + 2 + tid; b < n; b += nthr) Z[tt::xoff(a, b)] = __ldg(c + tri_c_index(layout, h, n, p, a, b));
         }
         __syncthreads();
         // 2. D = 0
         for (int I = tid; I < NT; I += nthr) {
-            T *r0 = Z + xc<3>(4 * I, I);
+            T *r0 = Z + xc(4 * I, I);
             const T4 c0 = tt::ld4(r0), c1 = tt::ld4(r0 + 4);
             const T z = T(0);
             const T t02 = Op::add(Op::add(z, z), c0.z);
@@ -856,7 +792,7 @@ tri_tiled_global_kernel(const T *__restrict__ c, T *__restrict__ out, T *ws, int
                     for (int v = 0; v < 4; ++v) acc[u][v] = Op::inf();
                 if (act) {
                     for (int m = I + 1 + q; m < J; m += s) {
-                        const T *pa = Z + xc<3>(4 * I, m), *pb = Z + xc<3>(4 * m, J);
+                        const T *pa = Z + xc(4 * I, m), *pb = Z + xc(4 * m, J);
                         T4 A[4], B[4];
 #pragma unroll
                         for (int u = 0; u < 4; ++u) A[u] = tt::ld4(pa + 4 * u), B[u] = tt::ld4(pb + 4 * u);
@@ -870,7 +806,7 @@ tri_tiled_global_kernel(const T *__restrict__ c, T *__restrict__ out, T *ws, int
                         for (int v = 0; v < 4; ++v)
                             acc[u][v] = Op::min(acc[u][v], __shfl_xor_sync(0xffffffffu, acc[u][v], off));
                 if (act && q == 0) {
-                    T *ta = Z + xc<3>(4 * I, I), *tb = Z + xc<3>(4 * J, J), *tc = Z + xc<3>(4 * I, J);
+                    T *ta = Z + xc(4 * I, I), *tb = Z + xc(4 * J, J), *tc = Z + xc(4 * I, J);
                     T A[4][4], Bd[4][4], C[4][4];
 #pragma unroll
                     for (int r = 0; r < 4; ++r) {
@@ -887,7 +823,7 @@ tri_tiled_global_kernel(const T *__restrict__ c, T *__restrict__ out, T *ws, int
             }
             __syncthreads();
         }
-        if (tid == 0) out[h] = Z[tt::xoff<3>(0, n - 1)];
+        if (tid == 0) out[h] = Z[tt::xoff(0, n - 1)];
     }
 }
 
@@ -896,7 +832,7 @@ int tiled_global_threads(int64_t n) { return n >= 256 ? 512 : 256; }
 size_t tiled_global_workspace(int64_t n, int64_t p) {
     const int NT = static_cast<int>((n + 3) / 4);
     const long long grid = std::min<long long>(p, num_sms());
-    return static_cast<size_t>(grid) * 4 * tt::colbase<3>(NT) * 4;
+    return static_cast<size_t>(grid) * 4 * tt::colbase(NT) * 4;
 }
 
 int launch_tri_tiled_global(const void *c, void *out, void *ws, int64_t n, int64_t p, int dtype, int layout,
