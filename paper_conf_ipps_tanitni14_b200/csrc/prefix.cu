@@ -104,14 +104,24 @@ template <int INST> struct Cfg {
 #ifndef BO_FR_STAGES
 #define BO_FR_STAGES 8      // measured: 1 CTA/SM with a 7-8 deep ring beats 2 CTAs x 6 (99.3 % vs 96.0 % of HBM)
 #endif
-    // 32-instance tiles serve small p (measured: a 24-deep ring is slower, n = 1024
-    // p = 16384 42 vs 23.5 us, n = 32K p = 8K 0.585 vs 0.555 ms: 2 CTAs/SM instead of 6)
+    // 32-instance tiles serve small p.  Chunks (TMA boxes) per ring stage: a stage's
+    // scan, barrier and stores are one dependent round of the CTA, so with 4 KiB
+    // boxes several chunks per stage keep that fixed cost off each box.  Measured
+    // (stages x chunks): 3 x 4 against 8 x 1 -- n = 32K p = 8K 0.477 vs 0.554 ms,
+    // n = 4096 p = 8192 65 vs 73 us, n = 1024 p = 4096 18.2 vs 20.9 us, p = 32768 48.7
+    // vs 50.5 us, p = 16384 23.9 vs 23.6 us; 4 x 4 and 6 x 4 lose at p = 16384 (34 us:
+    // fewer CTAs per SM than tiles), a 24 x 1 ring loses everywhere.
 #ifndef BO_FR_STAGES32
-#define BO_FR_STAGES32 8
+#define BO_FR_STAGES32 3
+#endif
+#ifndef BO_FR_CPS32
+#define BO_FR_CPS32 4
 #endif
     static constexpr int kStages = INST == 128 ? BO_FR_STAGES : BO_FR_STAGES32;
+    static constexpr int kCps = INST == 128 ? 1 : BO_FR_CPS32;
     static constexpr uint32_t kBoxBytes = INST * kElems * 4;   // 16 KiB / 4 KiB
-    static constexpr size_t kSmem = 1024 + kStages * kBoxBytes + kStages * 16;
+    static constexpr uint32_t kStageBytes = kCps * kBoxBytes;
+    static constexpr size_t kSmem = 1024 + kStages * kStageBytes + kStages * 20;
 };
 }  // namespace fr
 
@@ -124,13 +134,16 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
     pdl_begin();
     using fr::kElems;
     constexpr int kStages = fr::Cfg<kInst>::kStages;
+    constexpr int kCps = fr::Cfg<kInst>::kCps;
     constexpr uint32_t kBoxBytes = fr::Cfg<kInst>::kBoxBytes;
+    constexpr uint32_t kStageBytes = fr::Cfg<kInst>::kStageBytes;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                                ~uintptr_t(1023));
-    uint64_t *full = reinterpret_cast<uint64_t *>(buf + kStages * kBoxBytes);
+    uint64_t *full = reinterpret_cast<uint64_t *>(buf + kStages * kStageBytes);
     int *stage_tile = reinterpret_cast<int *>(full + kStages);    // tile of each ring slot, -1 = end
-    int *stage_chunk = stage_tile + kStages;
+    int *stage_chunk = stage_tile + kStages;                      // its first chunk
+    int *stage_cnt = stage_chunk + kStages;                       // and how many (<= kCps, one tile)
     WorkSlot *ws = slot >= 0 ? &g_fr_slots[slot] : nullptr;
     const int tid = threadIdx.x;
 
@@ -157,12 +170,15 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
             mbar_arrive(&full[s]);
             return;
         }
+        const int cnt = min(kCps, nchunks - prod_chunk);
         stage_tile[s] = static_cast<int>(prod_tile);
         stage_chunk[s] = prod_chunk;
-        mbar_arrive_expect_tx(&full[s], kBoxBytes);
-        tma_load_2d(buf + s * kBoxBytes, &src_map, prod_chunk * kElems, static_cast<int>(prod_tile * kInst),
-                    &full[s]);
-        ++prod_chunk;
+        stage_cnt[s] = cnt;
+        mbar_arrive_expect_tx(&full[s], cnt * kBoxBytes);
+        for (int b = 0; b < cnt; ++b)
+            tma_load_2d(buf + s * kStageBytes + b * kBoxBytes, &src_map, (prod_chunk + b) * kElems,
+                        static_cast<int>(prod_tile * kInst), &full[s]);
+        prod_chunk += cnt;
     };
     if (tid == 0)
         for (int s = 0; s < kStages - 1 && !prod_done; ++s) issue(s);
@@ -174,24 +190,30 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
         const int tile = stage_tile[s];
         if (tile < 0) break;
         const int chunk = stage_chunk[s];
+        const int cnt = kCps == 1 ? 1 : stage_cnt[s];
         if (chunk == 0) r = T(0);                       // new tile: r_j <- 0
-        uint8_t *box = buf + s * kBoxBytes;
 #pragma unroll
-        for (int k = 0; k < kElems / 4; ++k) {
-            uint4 *q = reinterpret_cast<uint4 *>(box + swz128(tid, k));
-            uint4 v = *q;
-            r = add_wrap(r, bits_as<T>(v.x)); v.x = as_bits(r);   // r <- r + b[i]; b[i] <- r
-            r = add_wrap(r, bits_as<T>(v.y)); v.y = as_bits(r);
-            r = add_wrap(r, bits_as<T>(v.z)); v.z = as_bits(r);
-            r = add_wrap(r, bits_as<T>(v.w)); v.w = as_bits(r);
-            *q = v;
+        for (int b = 0; b < kCps; ++b) {
+            if (kCps > 1 && b >= cnt) break;
+            uint8_t *box = buf + s * kStageBytes + b * kBoxBytes;
+#pragma unroll
+            for (int k = 0; k < kElems / 4; ++k) {
+                uint4 *q = reinterpret_cast<uint4 *>(box + swz128(tid, k));
+                uint4 v = *q;
+                r = add_wrap(r, bits_as<T>(v.x)); v.x = as_bits(r);   // r <- r + b[i]; b[i] <- r
+                r = add_wrap(r, bits_as<T>(v.y)); v.y = as_bits(r);
+                r = add_wrap(r, bits_as<T>(v.z)); v.z = as_bits(r);
+                r = add_wrap(r, bits_as<T>(v.w)); v.w = as_bits(r);
+                *q = v;
+            }
         }
         fence_proxy_async_smem();
         __syncthreads();
         if (tid == 0) {
-            tma_store_2d(&dst_map, box, chunk * kElems, tile * kInst);
+            for (int b = 0; b < cnt; ++b)
+                tma_store_2d(&dst_map, buf + s * kStageBytes + b * kBoxBytes, (chunk + b) * kElems, tile * kInst);
             bulk_commit();
-            bulk_wait_read<1>();                       // store i-1 no longer reads its stage
+            bulk_wait_read<1>();                       // stage i-1's stores no longer read it
             if (!prod_done) issue(static_cast<int>((i + kStages - 1) % kStages));
         }
     }
