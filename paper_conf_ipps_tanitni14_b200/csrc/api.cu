@@ -168,7 +168,7 @@ int launch_gen_prefix(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int
 int launch_gen_tri(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
 int launch_checksum(const void *, int64_t, int64_t, int64_t, int, uint64_t *, cudaStream_t);
 int launch_exec(const void *prog, int64_t t, void *mem, int64_t msize, int64_t p, int dtype, int layout, int nregs,
-                cudaStream_t st);
+                int nzero, cudaStream_t st);
 
 static constexpr int64_t kMaxElems = int64_t(1) << 40;
 
@@ -341,7 +341,12 @@ int bulk_execute(const int32_t *prog, int64_t t, void *prog_dev, size_t prog_dev
     if (!prog_dev || prog_dev_bytes < static_cast<size_t>(t) * 16 || !aligned16(prog_dev))
         return fail(BO_EINVAL, "execute: device program buffer must be 16-byte aligned and >= 16*t bytes");
     // the program is validated here, on the host: every register < nregs and
-    // every address < msize, so the kernel never leaves the instance memory
+    // every address < msize, so the kernel never leaves the instance memory.
+    // Registers start at 0: the kernel zeroes them only if some register is
+    // read before it is written (`uninit_read`).
+    uint64_t written = 0;
+    bool uninit_read = false;
+    auto use = [&](int32_t r) { if (!((written >> r) & 1)) uninit_read = true; };
     for (int64_t i = 0; i < t; ++i) {
         const int32_t op = prog[4 * i], x = prog[4 * i + 1], y = prog[4 * i + 2], z = prog[4 * i + 3];
         auto reg = [&](int32_t r) { return r >= 0 && r < nregs; };
@@ -356,12 +361,18 @@ int bulk_execute(const int32_t *prog, int64_t t, void *prog_dev, size_t prog_dev
             default: ok = false;
         }
         if (!ok) return fail(BO_EINVAL, "execute: bad instruction " + std::to_string(i));
+        switch (op) {                                      // reads, then the write
+            case 1: use(y); break;
+            case 2: case 3: case 4: case 5: use(y); use(z); written |= 1ull << x; break;
+            case 6: use(y); written |= 1ull << x; break;
+            default: written |= 1ull << x; break;      // LOAD, CONST
+        }
     }
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     int rc = cuda_check(cudaMemcpyAsync(prog_dev, prog, static_cast<size_t>(t) * 16, cudaMemcpyHostToDevice, st),
                         "execute: program upload");
     if (rc) return rc;
-    return launch_exec(prog_dev, t, mem, msize, p, dtype, layout, nregs, st);
+    return launch_exec(prog_dev, t, mem, msize, p, dtype, layout, nregs, uninit_read ? nregs : 0, st);
 }
 
 int bulk_triangulation_chords(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int dtype,

@@ -24,13 +24,16 @@ __device__ __forceinline__ float ex_sub(float a, float b) { return __fsub_rn(a, 
 
 template <typename T, int LAYOUT>
 __global__ void __launch_bounds__(ex::kThreads)
-exec_kernel(const int4 *__restrict__ prog, long long t, T *mem, long long msize, long long p) {
+exec_kernel(const int4 *__restrict__ prog, long long t, T *mem, long long msize, long long p, int nzero) {
     pdl_begin();
     extern __shared__ uint8_t smem_raw[];
     T *R = reinterpret_cast<T *>(smem_raw) + threadIdx.x;     // r[x] at R[x * kThreads]
     const long long j = blockIdx.x * static_cast<long long>(ex::kThreads) + threadIdx.x;
     const bool live = j < p;
     auto addr = [&](long long a) -> long long { return LAYOUT == BO_ROW_WISE ? j * msize + a : a * p + j; };
+    // registers start at 0 (bulkobl.h); the host passes nzero = 0 when the program
+    // writes every register before reading it (every builder in programs.py does)
+    for (int x = 0; x < nzero; ++x) R[x * ex::kThreads] = T(0);
     for (long long i = 0; i < t; ++i) {
         const int4 ins = __ldg(prog + i);                      // same address for the whole warp
         const int x = ins.y, y = ins.z, z = ins.w;
@@ -61,16 +64,16 @@ exec_kernel(const int4 *__restrict__ prog, long long t, T *mem, long long msize,
 }
 
 int launch_exec(const void *prog, int64_t t, void *mem, int64_t msize, int64_t p, int dtype, int layout, int nregs,
-                cudaStream_t st) {
+                int nzero, cudaStream_t st) {
     const size_t smem = static_cast<size_t>(nregs) * ex::kThreads * 4;
     const unsigned grid = static_cast<unsigned>((p + ex::kThreads - 1) / ex::kThreads);
     const int4 *pg = static_cast<const int4 *>(prog);
     if (dtype == BO_F32) {
-        if (layout == BO_ROW_WISE) launch(exec_kernel<float, BO_ROW_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<float *>(mem), msize, p);
-        else launch(exec_kernel<float, BO_COLUMN_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<float *>(mem), msize, p);
+        if (layout == BO_ROW_WISE) launch(exec_kernel<float, BO_ROW_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<float *>(mem), msize, p, nzero);
+        else launch(exec_kernel<float, BO_COLUMN_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<float *>(mem), msize, p, nzero);
     } else {
-        if (layout == BO_ROW_WISE) launch(exec_kernel<int32_t, BO_ROW_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<int32_t *>(mem), msize, p);
-        else launch(exec_kernel<int32_t, BO_COLUMN_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<int32_t *>(mem), msize, p);
+        if (layout == BO_ROW_WISE) launch(exec_kernel<int32_t, BO_ROW_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<int32_t *>(mem), msize, p, nzero);
+        else launch(exec_kernel<int32_t, BO_COLUMN_WISE>, grid, ex::kThreads, smem, st, pg, t, static_cast<int32_t *>(mem), msize, p, nzero);
     }
     return after_launch("exec_kernel");
 }
