@@ -154,8 +154,11 @@ def prefix_sums(x: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, ou
     dt = _dtype_code(x)
     if out is None:
         out = torch.empty_like(x)
-    _check_out(out, x, x.shape)
-    need = prefix_sums_workspace(n, p, dt, layout, variant)
+    else:
+        _check_out(out, x, x.shape)
+    # only the explicit-transpose variant uses a workspace (AUTO never resolves to it):
+    # skip the query, a ctypes round trip, on the hot small-call path
+    need = prefix_sums_workspace(n, p, dt, layout, variant) if variant == PS_TRANSPOSED else 0
     wptr, wbytes = None, 0
     if need:
         if workspace is None:
@@ -235,7 +238,8 @@ def triangulation(c: torch.Tensor, layout: int = ROW_WISE, variant: int = AUTO, 
     dt = _dtype_code(c)
     if out is None:
         out = torch.empty(p, dtype=c.dtype, device=c.device)
-    _check_out(out, c, (p,))
+    else:
+        _check_out(out, c, (p,))
     need = triangulation_workspace(n, p, dt, layout, variant)
     wptr, wbytes = None, 0
     if need:
