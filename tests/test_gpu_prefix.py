@@ -168,6 +168,16 @@ def test_column_wise_tma_ring_ragged(dt, n, p):
 
 
 @pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("n,p", [(96, 1000), (1060, 333), (4100, 64), (128, 37887), (32, 40)])
+def test_fused_row_32_instance_tiles_multi_box_stages(dt, n, p):
+    # the 32-instance fused-row tiles carry 4 TMA boxes per ring stage: chunk counts that are not a
+    # multiple of 4 (3, 34, 129 chunks), a ragged last tile, and a tile count below the SM count
+    x = bulkgen.prefix_input(n, p, seed=n + 3 * p, dtype=dt)
+    got = bo.prefix_sums(torch.from_numpy(x).to(DEV), bo.ROW_WISE, bo.PS_FUSED_ROW).cpu().numpy()
+    assert np.array_equal(got.view(np.uint32), oracle.bulk_prefix_sums(x, oracle.ROW_WISE).view(np.uint32))
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
 @pytest.mark.parametrize("n,p", [(256, 32), (300, 36), (1000, 4100), (257, 996), (4096, 132), (2000, 37884)])
 def test_column_wise_tma_ring_32_wide(dt, n, p):
     # the 32-instance column-block TMA ring (p % 4 == 0, p below 2*128*SMs, n >= 256): partial last
