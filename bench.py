@@ -695,6 +695,14 @@ def run_ours(args, ctx):
     # the oracle on a sample of rank 0's shard (before anything reuses st's buffers)
     if args.cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(ctx, name, st) if ctx.rank == 0 else None
+        cb = line["cpu_baseline"]
+        if cb and cb.get("single_core"):
+            # north_star: quote the paper's GPU-over-one-CPU factor as context only
+            line["speedup_context"] = {
+                "gpu_over_oracle_one_core": line["value"] / cb["single_core"]["value"],
+                "gpu_over_oracle_all_cores": line["value"] / cb["value"],
+                "paper": "more than 150x GPU (GTX Titan) over one Core i7 core at n=1K, p>=8K (P:249); "
+                         "context only -- another GPU, another CPU, another decade"}
     # G-invariance: rank 0 recomputes every rank's shard on its own GPU, one after
     # the other (what a single-GPU run of the whole problem computes), and compares
     if ctx.rank == 0 and wl["algo"] in ("prefix", "tri") and "fn_on" in st:
