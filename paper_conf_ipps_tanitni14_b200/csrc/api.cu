@@ -6,7 +6,6 @@
 #include <cstring>
 #include <mutex>
 #include <set>
-#include <thread>
 #include <string>
 #include <utility>
 #include <vector>
@@ -69,35 +68,36 @@ int work_slot_for(cudaStream_t st) {
     // A queue slot is reset by the last CTA of the launch that used it, so two
     // launches may share one only if the second cannot start before the first
     // has finished: launches on one stream (griddepcontrol.wait precedes every
-    // access to the slot).  So each (device, stream) owns a slot.  A launch
-    // being captured into a graph gets none (-1: static tile striding): the
-    // graph may be replayed on any stream, beside eager launches on this one.
+    // access to the slot).  So each (device, stream) owns a slot, keyed by the
+    // stream's process-unique id (cudaStreamGetId: a destroyed stream's handle
+    // may be reused while its work still runs; cudaStreamPerThread resolves to
+    // the calling thread's stream).  A launch being captured into a graph gets
+    // none (-1: static tile striding): the graph may be replayed on any stream,
+    // beside eager launches on this one.
     cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
     if (cudaStreamIsCapturing(st, &cap) != cudaSuccess) {
         cudaGetLastError();
         return -1;
     }
-    if (cap != cudaStreamCaptureStatusNone) return -1;
+    if (cap != cudaStreamCaptureStatusNone) return -1;   // (cudaStreamGetId would invalidate a capture)
+    unsigned long long sid = 0;
+    if (cudaStreamGetId(st, &sid) != cudaSuccess) {
+        cudaGetLastError();
+        return -1;
+    }
     int dev = 0;
     cudaGetDevice(&dev);
-    // cudaStreamPerThread is one handle for a different stream in every thread
-    const std::thread::id tid = st == cudaStreamPerThread ? std::this_thread::get_id() : std::thread::id();
-    struct Owner {
-        int dev;
-        cudaStream_t st;
-        std::thread::id tid;
-    };
     static std::mutex mu;
-    static std::vector<Owner> owners;                            // in order of first use
+    static std::vector<std::pair<int, unsigned long long>> owners;   // (device, stream id), first use order
     std::lock_guard<std::mutex> g(mu);
     int used_on_dev = 0;
-    for (const Owner &o : owners) {
-        if (o.dev != dev) continue;
-        if (o.st == st && o.tid == tid) return used_on_dev;
+    for (const auto &o : owners) {
+        if (o.first != dev) continue;
+        if (o.second == sid) return used_on_dev;
         ++used_on_dev;
     }
     if (used_on_dev >= kWorkSlots) return -1;                   // beyond 256 streams: static striding
-    owners.push_back(Owner{dev, st, tid});
+    owners.emplace_back(dev, sid);
     return used_on_dev;
 }
 

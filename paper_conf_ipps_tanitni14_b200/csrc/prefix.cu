@@ -170,15 +170,22 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
             mbar_arrive(&full[s]);
             return;
         }
-        const int cnt = min(kCps, nchunks - prod_chunk);
         stage_tile[s] = static_cast<int>(prod_tile);
         stage_chunk[s] = prod_chunk;
-        stage_cnt[s] = cnt;
-        mbar_arrive_expect_tx(&full[s], cnt * kBoxBytes);
-        for (int b = 0; b < cnt; ++b)
-            tma_load_2d(buf + s * kStageBytes + b * kBoxBytes, &src_map, (prod_chunk + b) * kElems,
-                        static_cast<int>(prod_tile * kInst), &full[s]);
-        prod_chunk += cnt;
+        if constexpr (kCps == 1) {
+            mbar_arrive_expect_tx(&full[s], kBoxBytes);
+            tma_load_2d(buf + s * kStageBytes, &src_map, prod_chunk * kElems, static_cast<int>(prod_tile * kInst),
+                        &full[s]);
+            ++prod_chunk;
+        } else {
+            const int cnt = min(kCps, nchunks - prod_chunk);
+            stage_cnt[s] = cnt;
+            mbar_arrive_expect_tx(&full[s], cnt * kBoxBytes);
+            for (int b = 0; b < cnt; ++b)
+                tma_load_2d(buf + s * kStageBytes + b * kBoxBytes, &src_map, (prod_chunk + b) * kElems,
+                            static_cast<int>(prod_tile * kInst), &full[s]);
+            prod_chunk += cnt;
+        }
     };
     if (tid == 0)
         for (int s = 0; s < kStages - 1 && !prod_done; ++s) issue(s);
@@ -210,8 +217,11 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
         fence_proxy_async_smem();
         __syncthreads();
         if (tid == 0) {
-            for (int b = 0; b < cnt; ++b)
+#pragma unroll
+            for (int b = 0; b < kCps; ++b) {
+                if (kCps > 1 && b >= cnt) break;
                 tma_store_2d(&dst_map, buf + s * kStageBytes + b * kBoxBytes, (chunk + b) * kElems, tile * kInst);
+            }
             bulk_commit();
             bulk_wait_read<1>();                       // stage i-1's stores no longer read it
             if (!prod_done) issue(static_cast<int>((i + kStages - 1) % kStages));
