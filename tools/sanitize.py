@@ -37,6 +37,22 @@ from paper_conf_ipps_tanitni14_b200 import programs  # noqa: E402
 for layout in (bo.ROW_WISE, bo.COLUMN_WISE):
     m = bo.generate_prefix(16, 70, 1, torch.float32, layout)
     bo.execute(programs.bitonic_sort(16), m, layout)
+# a program that reads registers before writing them (the kernel zeroes its register file)
+import numpy as np  # noqa: E402
+bo.execute(np.array([[2, 0, 1, 2], [1, 0, 0, 0]], dtype=np.int32), torch.zeros((64, 4), dtype=torch.int32,
+                                                                                 device="cuda"), bo.ROW_WISE)
+# graph capture: the queue kernels stride statically, eager launches on another stream beside it
+xg = bo.generate_prefix(1024, 40000, 3, torch.float32, bo.ROW_WISE)
+og = torch.empty_like(xg)
+sc = torch.cuda.Stream()
+with torch.cuda.stream(sc):
+    bo.prefix_sums(xg, bo.ROW_WISE, out=og, stream=sc)
+sc.synchronize()
+g = torch.cuda.CUDAGraph()
+with torch.cuda.graph(g, stream=sc):
+    bo.prefix_sums(xg, bo.ROW_WISE, out=og, stream=sc)
+g.replay()
+bo.prefix_sums(xg, bo.ROW_WISE)
 x = torch.zeros((300, 260), dtype=torch.int32, device="cuda")
 bo.transpose(x)
 torch.cuda.synchronize()
