@@ -27,3 +27,4 @@ for tool in memcheck racecheck synccheck; do
   timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize.py > $OUT/sanitizer_$tool.log 2>&1
   echo "sanitizer $tool rc=$?"
 done
+timeout 1200 python bench.py --sweep > $OUT/sweep.json 2> $OUT/sweep.err; echo "sweep rc=$?"
