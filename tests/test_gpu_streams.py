@@ -166,3 +166,28 @@ def test_out_tensor_is_validated():
         bo.triangulation(c, bo.ROW_WISE, out=torch.empty(49, dtype=torch.int32, device=DEV))
     with pytest.raises(ValueError):
         bo.triangulation(c, bo.ROW_WISE, out=torch.empty(50, dtype=torch.float32, device=DEV))
+
+
+def test_captured_helper_replays_many_small_calls():
+    # bo.Captured: a sequence of small bulk calls recorded once; replays give the eager results
+    xs = [bo.generate_prefix(32, 1024, 70 + k, torch.int32, bo.ROW_WISE) for k in range(8)]
+    c = bo.generate_tri(16, 256, 71, torch.int32, bo.ROW_WISE)
+    ys = [torch.empty_like(x) for x in xs]
+    oc = torch.empty(256, dtype=torch.int32, device=DEV)
+
+    def step(s):
+        for x, y in zip(xs, ys):
+            bo.prefix_sums(x, bo.ROW_WISE, out=y, stream=s)
+        bo.triangulation(c, bo.ROW_WISE, out=oc, stream=s)
+
+    cap = bo.Captured(step)
+    for y in ys:
+        y.zero_()
+    oc.zero_()
+    torch.cuda.synchronize()
+    for _ in range(3):
+        cap.replay()
+    torch.cuda.synchronize()
+    for x, y in zip(xs, ys):
+        assert torch.equal(y, bo.prefix_sums(x, bo.ROW_WISE))
+    assert torch.equal(oc, bo.triangulation(c, bo.ROW_WISE))
