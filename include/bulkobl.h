@@ -182,6 +182,28 @@ int bulk_execute(const int32_t *prog, int64_t t, void *prog_dev, size_t prog_dev
                  int64_t p, int dtype, int layout, int nregs, void *stream);
 
 /* ------------------------------------------------------------------------- */
+/* Prepared programs: validate, rewrite (the executor's internal              */
+/* superinstructions) and upload an oblivious program ONCE, then run it on    */
+/* any number of bulk memories with no per-call host work -- and inside CUDA  */
+/* graph capture, where bulk_execute can only upload the program unfused.     */
+/*   bulk_program_prepare: prog/t/msize/nregs as bulk_execute (same           */
+/*     validation, same BO_EINVAL messages); prog_dev: device buffer (16-byte */
+/*     aligned, >= 16*t bytes) that receives the rewritten program on         */
+/*     `stream` and must stay allocated and unmodified until release; the     */
+/*     host `prog` may be freed on return.  BO_EINVAL if `stream` is          */
+/*     capturing.  *handle receives a process-wide id (> 0).                  */
+/*   bulk_execute_prepared: runs the program on mem ([p][msize] row-wise or   */
+/*     [msize][p] column-wise, as bulk_execute); msize must equal the         */
+/*     prepared one; stream-ordered, capturable.  BO_EINVAL on an unknown     */
+/*     handle.                                                                */
+/*   bulk_program_release: forgets the handle (the caller frees prog_dev).    */
+/* ------------------------------------------------------------------------- */
+int bulk_program_prepare(const int32_t *prog, int64_t t, int64_t msize, int nregs, void *prog_dev,
+                         size_t prog_dev_bytes, void *stream, int64_t *handle);
+int bulk_execute_prepared(int64_t handle, void *mem, int64_t msize, int64_t p, int dtype, int layout, void *stream);
+int bulk_program_release(int64_t handle);
+
+/* ------------------------------------------------------------------------- */
 /* Layout transpose (row-wise <-> column-wise arrangement):        */
 /*   dst[c*rows + r] = src[r*cols + c],  0 <= r < rows, 0 <= c < cols.        */
 /* Row-wise [p][n] -> column-wise [n][p] is (rows=p, cols=n); the reverse is  */

@@ -65,6 +65,9 @@ def lib() -> ctypes.CDLL:
             "bulk_transpose": ([vp, vp, i64, i64, sz, vp], i32),
             "bulk_triangulation_chords": ([vp, vp, vp, i64, i64, i32, i32, vp], i32),
             "bulk_execute": ([vp, i64, vp, sz, vp, i64, i64, i32, i32, i32, vp], i32),
+            "bulk_program_prepare": ([vp, i64, i64, i32, vp, sz, vp, ctypes.POINTER(i64)], i32),
+            "bulk_execute_prepared": ([i64, vp, i64, i64, i32, i32, vp], i32),
+            "bulk_program_release": ([i64], i32),
             "bulk_prefix_sums_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_triangulation_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_prefix_sums_host_bytes": ([i64, i64, i32, i32, i32], sz),
@@ -272,18 +275,53 @@ def triangulation_chords(c: torch.Tensor, layout: int = ROW_WISE, stream=None, o
     return out, chords
 
 
-def execute(program, mem: torch.Tensor, layout: int = COLUMN_WISE, prog_buf: torch.Tensor | None = None,
-            stream=None) -> torch.Tensor:
-    """Bulk execution of an oblivious program (NEXT-3, Theorem 2 P:132-137) in
-    place on mem ([p, msize] row-wise or [msize, p] column-wise).  `program`
-    is a programs.Program or an int32 array [t, 4] (then nregs = 64)."""
+def _program_code(program):
     import numpy as np
-    _need_cuda(mem)
     if hasattr(program, "array"):
         code, nregs = program.array(), program.nregs
     else:
         code, nregs = np.asarray(program, dtype=np.int32).reshape(-1, 4), 64
-    code = np.ascontiguousarray(code, dtype=np.int32)
+    return np.ascontiguousarray(code, dtype=np.int32), nregs
+
+
+class Prepared:
+    """An oblivious program validated, rewritten and uploaded once
+    (bulk_program_prepare) for `msize`-word instance memories on `device`;
+    execute(prepared, mem, layout) then does no host work per call and can be
+    captured into a CUDA graph."""
+
+    def __init__(self, program, msize: int, device="cuda", stream=None):
+        code, self.nregs = _program_code(program)
+        self.msize, self.t = int(msize), code.shape[0]
+        self.buf = torch.empty(max(self.t, 1) * 16, dtype=torch.uint8, device=device)   # owned: lives with self
+        h = ctypes.c_int64(0)
+        _check(lib().bulk_program_prepare(code.ctypes.data, self.t, self.msize, self.nregs, self.buf.data_ptr(),
+                                          self.buf.numel(), _stream(stream, self.buf), ctypes.byref(h)))
+        self.handle = h.value
+
+    def __del__(self):
+        if getattr(self, "handle", 0) and _lib is not None:
+            _lib.bulk_program_release(self.handle)
+            self.handle = 0
+
+
+def prepare(program, msize: int, device="cuda", stream=None) -> Prepared:
+    return Prepared(program, msize, device, stream)
+
+
+def execute(program, mem: torch.Tensor, layout: int = COLUMN_WISE, prog_buf: torch.Tensor | None = None,
+            stream=None) -> torch.Tensor:
+    """Bulk execution of an oblivious program (NEXT-3, Theorem 2 P:132-137) in
+    place on mem ([p, msize] row-wise or [msize, p] column-wise).  `program`
+    is a programs.Program, an int32 array [t, 4] (then nregs = 64) or a
+    Prepared program (no per-call host work)."""
+    _need_cuda(mem)
+    if isinstance(program, Prepared):
+        msize, p = _shape_np(mem, layout)
+        _check(lib().bulk_execute_prepared(program.handle, mem.data_ptr(), msize, p, _dtype_code(mem), layout,
+                                           _stream(stream, mem)))
+        return mem
+    code, nregs = _program_code(program)
     t = code.shape[0]
     msize, p = _shape_np(mem, layout)
     if prog_buf is None:

@@ -8,6 +8,7 @@
 #include <set>
 #include <string>
 #include <utility>
+#include <map>
 #include <vector>
 
 namespace bo {
@@ -52,15 +53,19 @@ int max_blocks_per_sm(const void *func, int threads, size_t smem) {
 }
 
 bool ensure_dyn_smem(const void *func, int bytes) {
+    // the opt-in is a per-(device, kernel) maximum: only ever raise it (a kernel
+    // launched with several sizes, e.g. the executor's staged one, must not have
+    // a later smaller opt-in undo an earlier larger one)
     static std::mutex mu;
-    static std::set<std::pair<int, std::pair<const void *, int>>> done;
+    static std::map<std::pair<int, const void *>, int> set_to;
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess) return false;
-    const auto key = std::make_pair(dev, std::make_pair(func, bytes));
+    const auto key = std::make_pair(dev, func);
     std::lock_guard<std::mutex> g(mu);
-    if (done.count(key)) return true;
+    auto it = set_to.find(key);
+    if (it != set_to.end() && it->second >= bytes) return true;
     if (cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess) return false;
-    done.insert(key);
+    set_to[key] = bytes;
     return true;
 }
 
@@ -167,6 +172,7 @@ size_t tri_workspace(int64_t n, int64_t p, int variant);
 int launch_gen_prefix(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
 int launch_gen_tri(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
 int launch_checksum(const void *, int64_t, int64_t, int64_t, int, uint64_t *, cudaStream_t);
+std::vector<int32_t> exec_device_program(const int32_t *prog, int64_t t);
 int launch_exec(const void *prog, int64_t t, void *mem, int64_t msize, int64_t p, int dtype, int layout, int nregs,
                 int nzero, cudaStream_t st);
 
@@ -329,24 +335,14 @@ int bulk_triangulation(const void *c, void *out, int64_t n, int64_t p, int dtype
     return tri_dispatch(c, out, n, p, dtype, layout, v, workspace, static_cast<cudaStream_t>(stream));
 }
 
-int bulk_execute(const int32_t *prog, int64_t t, void *prog_dev, size_t prog_dev_bytes, void *mem, int64_t msize,
-                 int64_t p, int dtype, int layout, int nregs, void *stream) {
-    t_err.clear();
-    if (t < 0 || msize < 0 || p < 0) return fail(BO_EINVAL, "execute: t, msize and p must be >= 0");
-    if (!valid_dtype(dtype) || !valid_layout(layout)) return fail(BO_EINVAL, "execute: bad dtype or layout");
-    if (nregs < 1 || nregs > 64) return fail(BO_EINVAL, "execute: need 1 <= nregs <= 64");
-    if (msize > 0 && p > kMaxElems / msize) return fail(BO_EINVAL, "execute: msize*p too large");
-    if (t == 0 || p == 0) return BO_OK;
-    if (!prog || !mem) return fail(BO_EINVAL, "execute: NULL pointer");
-    if (!prog_dev || prog_dev_bytes < static_cast<size_t>(t) * 16 || !aligned16(prog_dev))
-        return fail(BO_EINVAL, "execute: device program buffer must be 16-byte aligned and >= 16*t bytes");
-    // the program is validated here, on the host: every register < nregs and
-    // every address < msize, so the kernel never leaves the instance memory.
-    // Registers start at 0: the kernel zeroes them only if some register is
-    // read before it is written (`uninit_read`).
+// Host validation of an oblivious program (bulk_execute / bulk_program_prepare):
+// every register < nregs and every address < msize, so the kernel never leaves
+// the instance memory.  Registers start at 0: *uninit_read tells whether some
+// register is read before it is written (then the kernel zeroes its file).
+static int exec_validate(const int32_t *prog, int64_t t, int64_t msize, int nregs, bool *uninit_read) {
     uint64_t written = 0;
-    bool uninit_read = false;
-    auto use = [&](int32_t r) { if (!((written >> r) & 1)) uninit_read = true; };
+    *uninit_read = false;
+    auto use = [&](int32_t r) { if (!((written >> r) & 1)) *uninit_read = true; };
     for (int64_t i = 0; i < t; ++i) {
         const int32_t op = prog[4 * i], x = prog[4 * i + 1], y = prog[4 * i + 2], z = prog[4 * i + 3];
         auto reg = [&](int32_t r) { return r >= 0 && r < nregs; };
@@ -368,11 +364,116 @@ int bulk_execute(const int32_t *prog, int64_t t, void *prog_dev, size_t prog_dev
             default: written |= 1ull << x; break;      // LOAD, CONST
         }
     }
+    return BO_OK;
+}
+
+static int exec_check_sizes(int64_t t, int64_t msize, int64_t p, int nregs) {
+    if (t < 0 || msize < 0 || p < 0) return fail(BO_EINVAL, "execute: t, msize and p must be >= 0");
+    if (nregs < 1 || nregs > 64) return fail(BO_EINVAL, "execute: need 1 <= nregs <= 64");
+    if (msize > 0 && p > kMaxElems / msize) return fail(BO_EINVAL, "execute: msize*p too large");
+    if (msize > INT32_MAX) return fail(BO_EINVAL, "execute: msize too large");
+    return BO_OK;
+}
+
+int bulk_execute(const int32_t *prog, int64_t t, void *prog_dev, size_t prog_dev_bytes, void *mem, int64_t msize,
+                 int64_t p, int dtype, int layout, int nregs, void *stream) {
+    t_err.clear();
+    if (int rc = exec_check_sizes(t, msize, p, nregs)) return rc;
+    if (!valid_dtype(dtype) || !valid_layout(layout)) return fail(BO_EINVAL, "execute: bad dtype or layout");
+    if (t == 0 || p == 0) return BO_OK;
+    if (!prog || !mem) return fail(BO_EINVAL, "execute: NULL pointer");
+    if (!prog_dev || prog_dev_bytes < static_cast<size_t>(t) * 16 || !aligned16(prog_dev))
+        return fail(BO_EINVAL, "execute: device program buffer must be 16-byte aligned and >= 16*t bytes");
+    bool uninit_read = false;
+    if (int rc = exec_validate(prog, t, msize, nregs, &uninit_read)) return rc;
     cudaStream_t st = static_cast<cudaStream_t>(stream);
-    int rc = cuda_check(cudaMemcpyAsync(prog_dev, prog, static_cast<size_t>(t) * 16, cudaMemcpyHostToDevice, st),
-                        "execute: program upload");
+    // Outside graph capture the uploaded program is the fused one (exec.cu:
+    // superinstructions; never longer than `prog`).  A captured copy node reads
+    // its host source at every replay, so under capture the caller's own `prog`
+    // is uploaded as it is (bulk_program_prepare gives a capturable fused one).
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    int rc = cuda_check(cudaStreamIsCapturing(st, &cap), "execute: stream");
     if (rc) return rc;
-    return launch_exec(prog_dev, t, mem, msize, p, dtype, layout, nregs, uninit_read ? nregs : 0, st);
+    std::vector<int32_t> fused;
+    const int32_t *up = prog;
+    int64_t tu = t;
+    if (cap == cudaStreamCaptureStatusNone) {
+        fused = exec_device_program(prog, t);
+        up = fused.data();
+        tu = static_cast<int64_t>(fused.size() / 4);
+    }
+    rc = cuda_check(cudaMemcpyAsync(prog_dev, up, static_cast<size_t>(tu) * 16, cudaMemcpyHostToDevice, st),
+                    "execute: program upload");
+    if (rc) return rc;
+    return launch_exec(prog_dev, tu, mem, msize, p, dtype, layout, nregs, uninit_read ? nregs : 0, st);
+}
+
+// ---- prepared programs: validated, fused and uploaded once
+namespace {
+struct PreparedProgram {
+    const void *dev;
+    int64_t tu, msize;
+    int nregs, nzero;
+};
+std::mutex g_prep_mu;
+std::map<int64_t, PreparedProgram> g_prep;
+int64_t g_prep_next = 1;
+}  // namespace
+
+int bulk_program_prepare(const int32_t *prog, int64_t t, int64_t msize, int nregs, void *prog_dev,
+                         size_t prog_dev_bytes, void *stream, int64_t *handle) {
+    t_err.clear();
+    if (!handle) return fail(BO_EINVAL, "prepare: NULL handle");
+    *handle = 0;
+    if (int rc = exec_check_sizes(t, msize, 0, nregs)) return rc;
+    if (t > 0 && !prog) return fail(BO_EINVAL, "prepare: NULL program");
+    if (!prog_dev || prog_dev_bytes < static_cast<size_t>(t) * 16 || !aligned16(prog_dev))
+        return fail(BO_EINVAL, "prepare: device program buffer must be 16-byte aligned and >= 16*t bytes");
+    bool uninit_read = false;
+    if (int rc = exec_validate(prog, t, msize, nregs, &uninit_read)) return rc;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    int rc = cuda_check(cudaStreamIsCapturing(st, &cap), "prepare: stream");
+    if (rc) return rc;
+    if (cap != cudaStreamCaptureStatusNone) return fail(BO_EINVAL, "prepare: not allowed while the stream is capturing");
+    const std::vector<int32_t> fused = exec_device_program(prog, t);
+    const int64_t tu = static_cast<int64_t>(fused.size() / 4);
+    if (tu > 0) {
+        // pageable source: the call returns once the words are staged, so the
+        // temporary may go; stream-ordered before any later launch on `stream`
+        rc = cuda_check(cudaMemcpyAsync(prog_dev, fused.data(), static_cast<size_t>(tu) * 16, cudaMemcpyHostToDevice, st),
+                        "prepare: program upload");
+        if (rc) return rc;
+    }
+    std::lock_guard<std::mutex> g(g_prep_mu);
+    const int64_t h = g_prep_next++;
+    g_prep[h] = PreparedProgram{prog_dev, tu, msize, nregs, uninit_read ? nregs : 0};
+    *handle = h;
+    return BO_OK;
+}
+
+int bulk_execute_prepared(int64_t handle, void *mem, int64_t msize, int64_t p, int dtype, int layout, void *stream) {
+    t_err.clear();
+    PreparedProgram pp;
+    {
+        std::lock_guard<std::mutex> g(g_prep_mu);
+        auto it = g_prep.find(handle);
+        if (it == g_prep.end()) return fail(BO_EINVAL, "execute_prepared: unknown program handle");
+        pp = it->second;
+    }
+    if (msize != pp.msize) return fail(BO_EINVAL, "execute_prepared: msize differs from the prepared program's");
+    if (int rc = exec_check_sizes(0, msize, p, pp.nregs)) return rc;
+    if (!valid_dtype(dtype) || !valid_layout(layout)) return fail(BO_EINVAL, "execute: bad dtype or layout");
+    if (pp.tu == 0 || p == 0) return BO_OK;
+    if (!mem) return fail(BO_EINVAL, "execute: NULL pointer");
+    return launch_exec(pp.dev, pp.tu, mem, msize, p, dtype, layout, pp.nregs, pp.nzero, static_cast<cudaStream_t>(stream));
+}
+
+int bulk_program_release(int64_t handle) {
+    t_err.clear();
+    std::lock_guard<std::mutex> g(g_prep_mu);
+    if (g_prep.erase(handle) == 0) return fail(BO_EINVAL, "release: unknown program handle");
+    return BO_OK;
 }
 
 int bulk_triangulation_chords(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int dtype,

@@ -50,8 +50,7 @@ def test_executor_rejects_bad_program():
 
 def _random_program(msize, nregs, t, seed, dt):
     """A random straight-line oblivious program: every op, random registers and
-    addresses, many STORE -> LOAD pairs on the same address inside the executor's
-    LOAD prefetch window (the host must mark those LOADs direct)."""
+    addresses, many STORE -> LOAD pairs on the same address a few instructions apart."""
     rng = np.random.default_rng(seed)
     code = []
     for _ in range(t):
@@ -73,10 +72,11 @@ def _random_program(msize, nregs, t, seed, dt):
 
 @pytest.mark.parametrize("dt", ["int32", "float32"])
 @pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
-@pytest.mark.parametrize("seed,t,msize", [(1, 40, 8), (2, 300, 16), (3, 1000, 12), (4, 5, 3), (5, 2000, 64)])
+@pytest.mark.parametrize("seed,t,msize", [(1, 40, 8), (2, 300, 16), (3, 1000, 12), (4, 5, 3), (5, 2000, 64),
+                                          (6, 1500, 400), (7, 900, 131)])
 def test_executor_random_programs_match_oracle(dt, layout, seed, t, msize):
-    # stresses the LOAD prefetch ring (exec.cu): loads of addresses stored a few instructions
-    # earlier, fewer LOADs than ring slots, registers read before any write (they start at 0)
+    # loads of addresses stored a few instructions earlier, registers read before any
+    # write (they start at 0)
     nregs = 7
     prog = _random_program(msize, nregs, t, seed, dt)
     p = 300
@@ -102,3 +102,144 @@ def test_executor_registers_start_at_zero():
     x = torch.full((64, 4), 7, dtype=torch.int32, device=DEV)
     bo.execute(prog, x, bo.ROW_WISE)
     assert torch.all(x[:, :2] == 0) and torch.all(x[:, 2:] == 7)
+
+
+def _fusable_program(msize, nregs, t, seed):
+    """Random programs made of the executor's superinstruction shapes (exec.cu: the
+    compare-exchange LOAD,LOAD,MIN,MAX,STORE,STORE and LOAD,OP,STORE), with register
+    and address collisions drawn often -- shapes that must fuse (either MIN/MAX
+    operand order, stores of any of the four registers, STORE over a loaded
+    address, both LOADs of one address) and near misses that must not (a register
+    shared between the loads and the results, MIN over a third register) -- mixed
+    with random single instructions."""
+    rng = np.random.default_rng(seed)
+    r = lambda: int(rng.integers(0, nregs))
+    a = lambda: int(rng.integers(0, min(msize, 4)))
+    code = []
+    while len(code) < t:
+        k = rng.random()
+        if k < 0.4:                                  # compare-exchange shape
+            ra, rb, rn, rx = (int(v) for v in rng.permutation(nregs)[:4])
+            if rng.random() < 0.2:                   # near miss: a collision
+                rn, rx = rng.choice([ra, rb, rn]), rng.choice([ra, rb, rx, rn])
+            y1, z1 = (ra, rb) if rng.random() < 0.5 else (rb, ra)
+            y2, z2 = (ra, rb) if rng.random() < 0.5 else (rb, ra)
+            if rng.random() < 0.1:
+                z1 = r()
+            q = lambda: int(rng.choice([ra, rb, rn, rx, r()]) if rng.random() < 0.9 else r())
+            code += [(0, ra, a(), 0), (0, rb, a(), 0), (4, rn, y1, z1), (5, rx, y2, z2),
+                     (1, a(), q(), 0), (1, a(), q(), 0)]
+        elif k < 0.55:                               # a run of in-place comparators (CE2 groups)
+            ra, rb, rn, rx = (int(v) for v in rng.permutation(nregs)[:4])
+            for _ in range(int(rng.integers(1, 10))):
+                A, B = (int(v) for v in rng.permutation(min(msize, 4))[:2])
+                y1, z1 = (ra, rb) if rng.random() < 0.5 else (rb, ra)
+                y2, z2 = (ra, rb) if rng.random() < 0.5 else (rb, ra)
+                code += [(0, ra, A, 0), (0, rb, B, 0), (4, rn, y1, z1), (5, rx, y2, z2),
+                         (1, A, rn, 0), (1, B, rx, 0)] if rng.random() < 0.5 else \
+                        [(0, ra, A, 0), (0, rb, B, 0), (4, rn, y1, z1), (5, rx, y2, z2),
+                         (1, B, rx, 0), (1, A, rn, 0)]
+        elif k < 0.7:                                # a run of accumulate steps (ACC_ADD groups)
+            acc, tmp = (int(v) for v in rng.permutation(nregs)[:2])
+            for _ in range(int(rng.integers(1, 20))):
+                yz = (acc, tmp) if rng.random() < 0.5 else (tmp, acc)
+                code += [(0, tmp, a(), 0), (2, acc, *yz), (1, a(), acc, 0)]
+        elif k < 0.8:                                # load-op-store shape, collisions likely
+            op = int(rng.integers(2, 6))
+            code += [(0, r(), a(), 0), (op, r(), r(), r()), (1, a(), r(), 0)]
+        else:
+            op = int(rng.choice([0, 1, 2, 3, 4, 5, 6]))
+            code.append((op, r(), a(), 0) if op == 0 else (op, a(), r(), 0) if op == 1 else (op, r(), r(), r()))
+    return np.asarray(code[:t], dtype=np.int32).reshape(-1, 4)
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("seed,t,nregs", [(11, 60, 5), (12, 600, 6), (13, 3000, 8), (14, 7, 4), (15, 2000, 64)])
+@pytest.mark.parametrize("msize", [9, 300])          # staged in shared memory / direct (exec_staged_smem)
+def test_executor_superinstruction_shapes_match_oracle(dt, layout, seed, t, nregs, msize):
+    prog = _fusable_program(msize, nregs, t, seed)
+    x = bulkgen.prefix_input(msize, 257 if msize < 100 else 1000, seed=seed, dtype=dt, layout=layout)
+    ref = oracle.bulk_execute(prog, x, layout)
+    got = torch.from_numpy(x).to(DEV)
+    bo.execute(prog, got, layout)
+    g = got.cpu().numpy()
+    if dt == "float32":
+        nan = np.isnan(g)
+        assert np.array_equal(nan, np.isnan(ref))
+        g, ref = g[~nan], ref[~nan]
+    assert np.array_equal(g.view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+def test_executor_captured_runs_unfused_program(layout):
+    # under graph capture the caller's program is uploaded as it is (api.cu)
+    n, p = 64, 300
+    P = programs.bitonic_sort(n)
+    x = bulkgen.prefix_input(n, p, seed=3, dtype="int32", layout=layout)
+    ref = oracle.bulk_execute(P.array(), x, layout)
+    buf = torch.from_numpy(x).to(DEV)
+    work = buf.clone()
+    prog_buf = torch.empty(P.array().shape[0] * 16, dtype=torch.uint8, device=DEV)
+    host = torch.from_numpy(P.array().copy()).pin_memory().numpy()   # read by the copy node at replay
+    g = bo.Captured(lambda s: (work.copy_(buf), bo.execute(host, work, layout, prog_buf=prog_buf, stream=s)))
+    g.replay()
+    torch.cuda.synchronize()
+    assert np.array_equal(work.cpu().numpy(), ref)
+
+
+def test_executor_alternating_shared_memory_sizes():
+    # the staged kernel's shared-memory opt-in is a per-kernel maximum: a large launch
+    # after a smaller one after a large one must still launch (api.cu ensure_dyn_smem)
+    outs = []
+    for msize in (120, 8, 120, 40, 120):
+        P = programs.bitonic_sort(8)
+        code = P.array().copy()
+        x = bulkgen.prefix_input(msize, 200, seed=msize, dtype="int32", layout=bo.COLUMN_WISE)
+        ref = oracle.bulk_execute(code, x, bo.COLUMN_WISE)
+        got = bo.execute(code, torch.from_numpy(x).to(DEV), bo.COLUMN_WISE).cpu().numpy()   # nregs 64
+        outs.append(np.array_equal(got, ref))
+    assert all(outs)
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("prog,n,p", [("prefix", 1024, 300), ("bitonic", 64, 1000), ("bitonic", 256, 130)])
+def test_prepared_program_matches_oracle(dt, layout, prog, n, p):
+    P = programs.prefix_sums(n, dt) if prog == "prefix" else programs.bitonic_sort(n)
+    prep = bo.prepare(P, n)
+    for seed in (1, 2):                                   # one preparation, several memories
+        x = bulkgen.prefix_input(n, p, seed=seed, dtype=dt, layout=layout)
+        ref = oracle.bulk_execute(P.array(), x, layout)
+        got = bo.execute(prep, torch.from_numpy(x).to(DEV), layout).cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.filterwarnings("ignore:The CUDA Graph is empty")       # the refused capture records nothing
+def test_prepared_program_checks_msize_and_capture():
+    P = programs.bitonic_sort(16)
+    prep = bo.prepare(P, 16)
+    with pytest.raises(bo.BulkError, match="msize"):
+        bo.execute(prep, torch.zeros((17, 8), dtype=torch.int32, device=DEV), bo.COLUMN_WISE)
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with pytest.raises(bo.BulkError, match="capturing"):
+        with torch.cuda.graph(g, stream=s):
+            bo.prepare(P, 16, stream=s)
+
+
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+def test_prepared_program_in_captured_graph(layout):
+    n, p = 64, 500
+    P = programs.bitonic_sort(n)
+    prep = bo.prepare(P, n)
+    x = bulkgen.prefix_input(n, p, seed=8, dtype="float32", layout=layout)
+    ref = oracle.bulk_execute(P.array(), x, layout)
+    src = torch.from_numpy(x).to(DEV)
+    work = torch.empty_like(src)
+    g = bo.Captured(lambda s: (work.copy_(src), bo.execute(prep, work, layout, stream=s)))
+    for _ in range(2):
+        work.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        assert np.array_equal(work.cpu().numpy(), ref)

@@ -145,3 +145,19 @@ def test_execute_validates_program_on_host(L):
     assert L.bulk_execute(good.ctypes.data, 2, p, 16, p, 8, 4, 0, 0, 4, None) == -1   # program buffer too small
     assert L.bulk_execute(good.ctypes.data, 2, p, 32, p, 8, 4, 0, 0, 0, None) == -1   # nregs = 0
     assert L.bulk_execute(good.ctypes.data, 0, p, 32, p, 8, 4, 0, 0, 4, None) == 0    # empty program
+
+
+def test_program_prepare_validates_on_host(L):
+    import numpy as np
+    p = ctypes.c_void_p(4096)
+    h = ctypes.c_int64(7)
+    for bad in ([[0, 0, 8, 0]], [[1, 0, 9, 0]], [[14, 0, 0, 0]]):     # internal opcodes are not accepted either
+        prog = np.array(bad, dtype=np.int32)
+        assert L.bulk_program_prepare(prog.ctypes.data, 1, 8, 4, p, 16, None, ctypes.byref(h)) == -1
+        assert b"bad instruction 0" in L.bulk_last_error() and h.value == 0
+    good = np.array([[0, 0, 3, 0], [1, 3, 0, 0]], dtype=np.int32)
+    assert L.bulk_program_prepare(good.ctypes.data, 2, 8, 4, p, 16, None, ctypes.byref(h)) == -1   # buffer small
+    assert L.bulk_program_prepare(good.ctypes.data, 2, 8, 4, p, 32, None, None) == -1               # NULL handle
+    assert L.bulk_execute_prepared(123456, p, 8, 4, 0, 0, None) == -1
+    assert b"unknown program handle" in L.bulk_last_error()
+    assert L.bulk_program_release(123456) == -1

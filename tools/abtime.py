@@ -2,7 +2,8 @@
 """Development A/B timer: time bench.py workloads exactly as bench.py does
 (rotating input copies, spin kernel ahead of the events, K steps back to back)
 for the library BULKOBL_LIB points at.  One JSON line per workload.
-    BULKOBL_LIB=ab/NAME/libbulkobl.so python tools/abtime.py ps2col tr2 prefix:1024:16384:float32:0 [--steps 20] [--reps 3]"""
+    BULKOBL_LIB=ab/NAME/libbulkobl.so python tools/abtime.py ps2col tr2 prefix:1024:16384:float32:0 [--steps 20] [--reps 3]
+(ad-hoc executor specs: exec_prefix:n:p:dtype:layout, exec_bitonic:n:p:dtype:layout)"""
 import json
 import os
 import sys
@@ -28,6 +29,8 @@ def main():
             f = name.split(":")
             wl = dict(seed=5, algo=f[0], n=int(f[1]), p=int(f[2]), dtype=f[3], layout=int(f[4]),
                       variant=int(f[5]) if len(f) > 5 else 0, desc=name)
+            if f[0].startswith("exec_"):              # exec_prefix:... / exec_bitonic:...
+                wl.update(algo="exec", prog=f[0][5:])
         else:
             wl = bench.WORKLOADS[name]
         st = bench.setup_workload(wl, 0, bench.copies_for(wl))

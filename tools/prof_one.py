@@ -1,5 +1,6 @@
 #!/usr/bin/env python
-"""Run one op a few times (for ncu).  python tools/prof_one.py prefix|tri|transpose n p dtype layout variant [reps]"""
+"""Run one op a few times (for ncu).
+    python tools/prof_one.py prefix|tri|transpose|exec_prefix|exec_bitonic n p dtype layout variant [reps]"""
 import os
 import sys
 
@@ -27,6 +28,12 @@ elif algo == "tri":
     ws = torch.empty(max(need, 1), dtype=torch.uint8, device="cuda")
     for _ in range(reps):
         bo.triangulation(c, layout, variant, out=o, workspace=ws)
+elif algo.startswith("exec_"):
+    from paper_conf_ipps_tanitni14_b200 import programs
+    P = programs.prefix_sums(n, sys.argv[4]) if algo == "exec_prefix" else programs.bitonic_sort(n)
+    x = bo.generate_prefix(n, p, 2, dt, layout)
+    for _ in range(reps):
+        bo.execute(P, x, layout)
 else:
     x = torch.empty((p, n), dtype=dt, device="cuda")
     for _ in range(reps):

@@ -36,7 +36,9 @@ for layout in (bo.COLUMN_WISE, bo.PACKED_ROW):
 from paper_conf_ipps_tanitni14_b200 import programs  # noqa: E402
 for layout in (bo.ROW_WISE, bo.COLUMN_WISE):
     m = bo.generate_prefix(16, 70, 1, torch.float32, layout)
-    bo.execute(programs.bitonic_sort(16), m, layout)
+    bo.execute(programs.bitonic_sort(16), m, layout)                     # staged in shared memory
+    bo.execute(programs.prefix_sums(300, "float32"), bo.generate_prefix(300, 130, 2, torch.float32, layout),
+               layout)                                                    # direct (msize too large to stage)
 # a program that reads registers before writing them (the kernel zeroes its register file)
 import numpy as np  # noqa: E402
 bo.execute(np.array([[2, 0, 1, 2], [1, 0, 0, 0]], dtype=np.int32), torch.zeros((64, 4), dtype=torch.int32,
