@@ -86,6 +86,8 @@ WORKLOADS = {
                              variant=0, desc="NEXT-3: generic executor, bitonic sort n=64, row-wise (Thm 2)"),
     "exec_prefix_col": dict(seed=2, algo="exec", prog="prefix", n=1024, p=2 ** 20, dtype="float32", layout=1,
                             variant=0, desc="NEXT-3: generic executor running Algorithm Prefix-sums, column-wise"),
+    "exec_prefix_row": dict(seed=2, algo="exec", prog="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0,
+                            variant=0, desc="NEXT-3: generic executor running Algorithm Prefix-sums, row-wise, windowed in shared memory"),
     # the paper's other experiment shapes (§V): n = 32K floats at p = 8K, 8-gons at
     # p = 4M, our kernels beside the paper's naive row-/column-wise kernels (Figs. 11, 12)
     "ps32k": dict(seed=21, algo="prefix", n=32768, p=8192, dtype="float32", layout=0, variant=0,
@@ -108,7 +110,7 @@ WORKLOADS = {
                          desc="the paper's row-wise kernel (thread per instance, uncoalesced)"),
 }
 EXTRAS = ["ps2col", "ps2tr", "tr_transpose", "ps1", "tr1", "tr1col", "tr1packed", "tr2", "tr2col", "tr2packed", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
-          "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col",
+          "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col", "exec_prefix_row",
           "ps32k", "ps32k_col", "ps32k_naive_row", "ps32k_naive_col", "tr8", "tr8col", "tr8_umm_row", "tr8_umm_col"]
 # The paper's own fitted GTX Titan models, in ms for p instances: context for the
 # extras of the same shape, never a target (another machine, another decade)

@@ -24,9 +24,13 @@ def sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")))
 
 
+def headers():
+    return sorted(glob.glob(os.path.join(CSRC, "*.cuh")) + glob.glob(os.path.join(CSRC, "*.h"))) + [
+        os.path.join(os.path.dirname(HERE), "include", "bulkobl.h")]
+
+
 def deps():
-    return sources() + sorted(glob.glob(os.path.join(CSRC, "*.cuh"))) + [
-        os.path.join(os.path.dirname(HERE), "include", "bulkobl.h"), __file__]
+    return sources() + headers() + [__file__]
 
 
 def up_to_date() -> bool:
@@ -54,8 +58,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
         objs.append(obj)
         if not force and os.path.exists(obj) and os.path.getmtime(obj) >= max(
-                os.path.getmtime(d) for d in [src] + sorted(glob.glob(os.path.join(CSRC, "*.cuh")))
-                + [os.path.join(os.path.dirname(HERE), "include", "bulkobl.h")]):
+                os.path.getmtime(d) for d in [src] + headers()):
             continue
         cmd = [NVCC, *FLAGS, "-c", src, "-o", obj]
         if verbose:

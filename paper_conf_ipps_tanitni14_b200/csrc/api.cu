@@ -2,6 +2,7 @@
 // validation, variant resolution, stream-ordered launches, and the pipelined
 // host-buffer entry points.  No computation happens on the CPU.
 #include "common.cuh"
+#include "exec.h"
 
 #include <cstring>
 #include <mutex>
@@ -172,9 +173,7 @@ size_t tri_workspace(int64_t n, int64_t p, int variant);
 int launch_gen_prefix(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
 int launch_gen_tri(void *, int64_t, int64_t, int64_t, uint64_t, int, int, int, cudaStream_t);
 int launch_checksum(const void *, int64_t, int64_t, int64_t, int, uint64_t *, cudaStream_t);
-std::vector<int32_t> exec_device_program(const int32_t *prog, int64_t t);
-int launch_exec(const void *prog, int64_t t, void *mem, int64_t msize, int64_t p, int dtype, int layout, int nregs,
-                int nzero, cudaStream_t st);
+
 
 static constexpr int64_t kMaxElems = int64_t(1) << 40;
 
@@ -394,18 +393,18 @@ int bulk_execute(const int32_t *prog, int64_t t, void *prog_dev, size_t prog_dev
     cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
     int rc = cuda_check(cudaStreamIsCapturing(st, &cap), "execute: stream");
     if (rc) return rc;
-    std::vector<int32_t> fused;
+    ExecProgram ep{{}, 0};
     const int32_t *up = prog;
     int64_t tu = t;
     if (cap == cudaStreamCaptureStatusNone) {
-        fused = exec_device_program(prog, t);
-        up = fused.data();
-        tu = static_cast<int64_t>(fused.size() / 4);
+        ep = exec_device_program(prog, t, msize, nregs);
+        up = ep.words.data();
+        tu = static_cast<int64_t>(ep.words.size() / 4);
     }
     rc = cuda_check(cudaMemcpyAsync(prog_dev, up, static_cast<size_t>(tu) * 16, cudaMemcpyHostToDevice, st),
                     "execute: program upload");
     if (rc) return rc;
-    return launch_exec(prog_dev, tu, mem, msize, p, dtype, layout, nregs, uninit_read ? nregs : 0, st);
+    return launch_exec(prog_dev, tu, mem, msize, p, dtype, layout, nregs, uninit_read ? nregs : 0, ep.wmax, st);
 }
 
 // ---- prepared programs: validated, fused and uploaded once
@@ -413,7 +412,7 @@ namespace {
 struct PreparedProgram {
     const void *dev;
     int64_t tu, msize;
-    int nregs, nzero;
+    int nregs, nzero, wmax;
 };
 std::mutex g_prep_mu;
 std::map<int64_t, PreparedProgram> g_prep;
@@ -436,7 +435,8 @@ int bulk_program_prepare(const int32_t *prog, int64_t t, int64_t msize, int nreg
     int rc = cuda_check(cudaStreamIsCapturing(st, &cap), "prepare: stream");
     if (rc) return rc;
     if (cap != cudaStreamCaptureStatusNone) return fail(BO_EINVAL, "prepare: not allowed while the stream is capturing");
-    const std::vector<int32_t> fused = exec_device_program(prog, t);
+    const ExecProgram ep = exec_device_program(prog, t, msize, nregs);
+    const std::vector<int32_t> &fused = ep.words;
     const int64_t tu = static_cast<int64_t>(fused.size() / 4);
     if (tu > 0) {
         // pageable source: the call returns once the words are staged, so the
@@ -447,7 +447,7 @@ int bulk_program_prepare(const int32_t *prog, int64_t t, int64_t msize, int nreg
     }
     std::lock_guard<std::mutex> g(g_prep_mu);
     const int64_t h = g_prep_next++;
-    g_prep[h] = PreparedProgram{prog_dev, tu, msize, nregs, uninit_read ? nregs : 0};
+    g_prep[h] = PreparedProgram{prog_dev, tu, msize, nregs, uninit_read ? nregs : 0, ep.wmax};
     *handle = h;
     return BO_OK;
 }
@@ -466,7 +466,8 @@ int bulk_execute_prepared(int64_t handle, void *mem, int64_t msize, int64_t p, i
     if (!valid_dtype(dtype) || !valid_layout(layout)) return fail(BO_EINVAL, "execute: bad dtype or layout");
     if (pp.tu == 0 || p == 0) return BO_OK;
     if (!mem) return fail(BO_EINVAL, "execute: NULL pointer");
-    return launch_exec(pp.dev, pp.tu, mem, msize, p, dtype, layout, pp.nregs, pp.nzero, static_cast<cudaStream_t>(stream));
+    return launch_exec(pp.dev, pp.tu, mem, msize, p, dtype, layout, pp.nregs, pp.nzero, pp.wmax,
+                       static_cast<cudaStream_t>(stream));
 }
 
 int bulk_program_release(int64_t handle) {

@@ -41,7 +41,11 @@
 //         GPU's NaN result carries no operand payload.
 #include "common.cuh"
 
+#include <algorithm>
+#include <climits>
 #include <vector>
+
+#include "exec.h"
 
 namespace bo {
 
@@ -54,20 +58,37 @@ namespace bo {
 #ifndef BO_EX_ACC_GROUP
 #define BO_EX_ACC_GROUP 8
 #endif
+#ifndef BO_EX_WINDOW_COL
+#define BO_EX_WINDOW_COL 0
+#endif
 #ifndef BO_EX_CE_GROUP
 #define BO_EX_CE_GROUP 2
 #endif
 
 namespace ex {
-enum { LOAD = 0, STORE, ADD, SUB, MIN, MAX, MOV, CONST, CE, LOS_ADD, LOS_SUB, LOS_MIN, LOS_MAX, CE2, ACC_ADD };
+enum { LOAD = 0, STORE, ADD, SUB, MIN, MAX, MOV, CONST, CE, LOS_ADD, LOS_SUB, LOS_MIN, LOS_MAX, CE2, ACC_ADD, WIN };
 constexpr int kThreads = 128;
+constexpr int kPitch = kThreads + 1;
+}
+
+// Shared memory of the staged kernel (0: run direct).  The cap keeps >= 3 CTAs
+// (12 warps) per SM.
+size_t exec_staged_smem(int64_t msize, int nregs) {
+    const size_t b = (static_cast<size_t>(nregs) * ex::kThreads + static_cast<size_t>(msize) * ex::kPitch) * 4;
+    return msize > 0 && b <= 72 * 1024 ? b : 0;
+}
+
+// Windowed staging: words of a window, so registers + window fit 64 KB (>= 3 CTAs per SM)
+static int exec_window_cap(int nregs) {
+    const int w = (64 * 1024 / 4 - nregs * ex::kThreads) / ex::kPitch;
+    return w < 64 ? w : 64;
 }
 
 // ---- host: the uploaded program (patterns above fused; the rest verbatim)
 // Registers are not observable after the program (only memory is), so a fused
 // instruction writes back only the registers a later instruction reads before
 // overwriting them: live_after[i] = registers live after original instruction i.
-std::vector<int32_t> exec_device_program(const int32_t *prog, int64_t t) {
+static std::vector<int32_t> exec_fuse(const int32_t *prog, int64_t t) {
     auto op = [&](int64_t i) { return i < t ? prog[4 * i] : -1; };
     auto f = [&](int64_t i, int k) { return prog[4 * i + k]; };
     std::vector<uint64_t> live_after(static_cast<size_t>(t));
@@ -145,6 +166,89 @@ std::vector<int32_t> exec_device_program(const int32_t *prog, int64_t t) {
     return out;
 }
 
+// Windows (instance memories too large to stage whole, exec_staged_smem == 0):
+// the fused program is cut greedily into segments whose addresses span at most
+// exec_window_cap words, each preceded by WIN (15, lo, len, 0); the kernel then
+// keeps [lo, lo+len) of its 128 instances in shared memory, copying it in (and
+// the previous window out, if stored to) with coalesced row segments.  Used
+// only when every instruction fits a window and the copies move at most twice
+// the words the program's own LOADs and STOREs touch (so a program that jumps
+// around its memory keeps the direct path).
+ExecProgram exec_device_program(const int32_t *prog, int64_t t, int64_t msize, int nregs) {
+    ExecProgram ep;
+    ep.words = exec_fuse(prog, t);
+    ep.wmax = 0;
+    if (msize <= 0 || exec_staged_smem(msize, nregs) != 0) return ep;
+    const int cap = exec_window_cap(nregs);
+    if (cap < 8) return ep;
+    const std::vector<int32_t> &w = ep.words;
+    const size_t nw = w.size() / 4;
+    // addresses of fused word i (second word of CE handled with its first)
+    struct Seg { size_t begin, end; int lo, hi; };
+    std::vector<Seg> segs;
+    long long direct = 0, copies = 0;
+    Seg cur{0, 0, INT32_MAX, -1};
+    bool stores = false;
+    auto close = [&](size_t end) {
+        cur.end = end;
+        if (cur.hi >= cur.lo) copies += static_cast<long long>(cur.hi - cur.lo + 1) * (stores ? 2 : 1);
+        segs.push_back(cur);
+        stores = false;
+    };
+    for (size_t i = 0; i < nw;) {
+        const int o = w[4 * i];
+        int a[4], na = 0, nst = 0;
+        size_t len = 1;
+        switch (o) {
+            case ex::LOAD: a[na++] = w[4 * i + 2]; break;
+            case ex::STORE: a[na++] = w[4 * i + 1]; nst = 1; break;
+            case ex::CE: a[na++] = w[4 * i + 1]; a[na++] = w[4 * i + 2]; a[na++] = w[4 * i + 4];
+                         a[na++] = w[4 * i + 5]; nst = 2; len = 2; break;
+            case ex::LOS_ADD: case ex::LOS_SUB: case ex::LOS_MIN: case ex::LOS_MAX:
+            case ex::ACC_ADD: a[na++] = w[4 * i + 1]; a[na++] = w[4 * i + 2]; nst = 1; break;
+            case ex::CE2: a[na++] = w[4 * i + 1]; a[na++] = w[4 * i + 2]; nst = 2; break;
+            default: break;
+        }
+        int lo = cur.lo, hi = cur.hi, ilo = INT32_MAX, ihi = -1;
+        for (int k = 0; k < na; ++k) {
+            ilo = std::min(ilo, a[k]);
+            ihi = std::max(ihi, a[k]);
+        }
+        if (na > 0 && ihi - ilo + 1 > cap) { ep.wmax = 0; return ep; }   // one instruction spans too much
+        if (na > 0) {
+            lo = std::min(lo, ilo);
+            hi = std::max(hi, ihi);
+            if (hi - lo + 1 > cap) {                                     // start a new window here
+                close(i);
+                cur = Seg{i, 0, ilo, ihi};
+            } else {
+                cur.lo = lo;
+                cur.hi = hi;
+            }
+            direct += na;
+            stores = stores || nst > 0;
+        }
+        i += len;
+    }
+    close(nw);
+    // worth it only with enough work per window, and never longer than the
+    // caller's program (the device buffer holds 16*t bytes)
+    if (copies > 2 * direct || static_cast<long long>(segs.size()) * 8 > direct ||
+        ep.words.size() + 4 * segs.size() > static_cast<size_t>(4 * t))
+        return ep;
+    std::vector<int32_t> out;
+    out.reserve(w.size() + 4 * segs.size());
+    for (const Seg &sg : segs) {
+        if (sg.hi >= sg.lo) {
+            out.insert(out.end(), {ex::WIN, sg.lo, sg.hi - sg.lo + 1, 0});
+            ep.wmax = std::max(ep.wmax, sg.hi - sg.lo + 1);
+        }
+        out.insert(out.end(), w.begin() + 4 * sg.begin, w.begin() + 4 * sg.end);
+    }
+    ep.words.swap(out);
+    return ep;
+}
+
 template <typename T>
 __device__ __forceinline__ T ex_add(T a, T b) { return add_wrap(a, b); }
 __device__ __forceinline__ int32_t ex_sub(int32_t a, int32_t b) {
@@ -159,15 +263,21 @@ __device__ __forceinline__ float ex_sub(float a, float b) { return __fsub_rn(a, 
 // coalesced loads, interprets against it, and copies every word back -- the
 // row-wise arrangement then costs what the column-wise one does (P:122-126's
 // difference is paid once, coalesced, instead of on every access).
-template <typename T, int LAYOUT, bool STAGED>
+// WINDOWED: the same for the window [wlo, wlo + wlen) the last WIN named.
+enum { EX_DIRECT = 0, EX_STAGED = 1, EX_WINDOWED = 2 };
+
+template <typename T, int LAYOUT, int MODE>
 __global__ void __launch_bounds__(ex::kThreads)
 exec_kernel(const int4 *__restrict__ prog, long long t, T *mem, long long msize, long long p, int nregs, int nzero) {
     pdl_begin();
+    constexpr bool STAGED = MODE == EX_STAGED;
     extern __shared__ uint8_t smem_raw[];
     T *R = reinterpret_cast<T *>(smem_raw) + threadIdx.x;     // r[x] at R[x * kThreads]
     T *Mb = reinterpret_cast<T *>(smem_raw) + nregs * ex::kThreads;
-    constexpr int kPitch = ex::kThreads + 1;
+    constexpr int kPitch = ex::kPitch;
     T *M = Mb + threadIdx.x;                                    // staged b[a] at M[a * kPitch]
+    int wlo = 0, wlen = 0;                                      // WINDOWED: current window
+    bool dirty = false;
     const long long j0 = blockIdx.x * static_cast<long long>(ex::kThreads);
     const long long j = j0 + threadIdx.x;
     const bool live = j < p;
@@ -176,11 +286,48 @@ exec_kernel(const int4 *__restrict__ prog, long long t, T *mem, long long msize,
     auto addr = [&](long long a) -> long long { return LAYOUT == BO_ROW_WISE ? j * msize + a : a * p + j; };
     auto ld = [&](int a) -> T {
         if constexpr (STAGED) return M[a * kPitch];
+        else if constexpr (MODE == EX_WINDOWED) return M[(a - wlo) * kPitch];
         else return live ? mem[addr(a)] : T(0);
     };
     auto st = [&](int a, T v) {
         if constexpr (STAGED) M[a * kPitch] = v;
+        else if constexpr (MODE == EX_WINDOWED) { M[(a - wlo) * kPitch] = v; dirty = true; }
         else if (live) mem[addr(a)] = v;
+    };
+    // WINDOWED: copy the window out / in, coalesced (row-wise: one warp per
+    // instance row segment; column-wise: one warp per address row)
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    auto window_out = [&]() {
+        if (LAYOUT == BO_ROW_WISE) {
+            for (int jl = warp; jl < cnt; jl += ex::kThreads / 32) {
+                T *g = mem + (j0 + jl) * msize + wlo;
+                for (int a = lane; a < wlen; a += 32) g[a] = Mb[a * kPitch + jl];
+            }
+        } else {
+            for (int a = 0; a < wlen; ++a)
+                if (live) mem[(wlo + a) * p + j] = M[a * kPitch];
+        }
+    };
+    auto window_in = [&]() {
+        if (LAYOUT == BO_ROW_WISE) {
+            // all of a thread's loads first (up to 2 x 32 in flight), then the stores
+            constexpr int kRows = ex::kThreads / (ex::kThreads / 32);   // 32 instance rows per warp
+            for (int a0 = 0; a0 < wlen; a0 += 32) {
+                const int a = a0 + lane;
+                T v[kRows];
+#pragma unroll
+                for (int r = 0; r < kRows; ++r) {
+                    const int jl = warp + r * (ex::kThreads / 32);
+                    v[r] = jl < cnt && a < wlen ? mem[(j0 + jl) * msize + wlo + a] : T(0);
+                }
+#pragma unroll
+                for (int r = 0; r < kRows; ++r)
+                    if (a < wlen) Mb[a * kPitch + warp + r * (ex::kThreads / 32)] = v[r];
+            }
+        } else {
+#pragma unroll 8
+            for (int a = 0; a < wlen; ++a) M[a * kPitch] = live ? mem[(wlo + a) * p + j] : T(0);
+        }
     };
     if constexpr (STAGED) {
         if (LAYOUT == BO_ROW_WISE) {                            // cnt*msize contiguous words
@@ -335,6 +482,17 @@ exec_kernel(const int4 *__restrict__ prog, long long t, T *mem, long long msize,
                 break;
             }
             case ex::MOV: R[x * ex::kThreads] = R[y * ex::kThreads]; break;
+            case ex::WIN:                                       // (15, lo, len): switch windows
+                if constexpr (MODE == EX_WINDOWED) {
+                    __syncthreads();
+                    if (dirty) window_out();
+                    wlo = x;
+                    wlen = y;
+                    dirty = false;
+                    window_in();
+                    __syncthreads();
+                }
+                break;
             case ex::CONST: {
                 const uint32_t u = static_cast<uint32_t>(y);
                 R[x * ex::kThreads] = *reinterpret_cast<const T *>(&u);
@@ -383,6 +541,10 @@ exec_kernel(const int4 *__restrict__ prog, long long t, T *mem, long long msize,
         }
         ++i;
     }
+    if constexpr (MODE == EX_WINDOWED) {
+        __syncthreads();
+        if (dirty) window_out();
+    }
     if constexpr (STAGED) {
         __syncthreads();
         if (LAYOUT == BO_ROW_WISE) {
@@ -399,35 +561,33 @@ exec_kernel(const int4 *__restrict__ prog, long long t, T *mem, long long msize,
     }
 }
 
-// Shared memory of the staged kernel (0: run direct).  The cap keeps >= 3 CTAs
-// (12 warps) per SM.
-size_t exec_staged_smem(int64_t msize, int nregs) {
-    const size_t b = (static_cast<size_t>(nregs) * ex::kThreads + static_cast<size_t>(msize) * (ex::kThreads + 1)) * 4;
-    return msize > 0 && b <= 72 * 1024 ? b : 0;
-}
-
 template <typename T, int LAYOUT>
 static void launch_exec_t(const int4 *pg, int64_t t, T *mem, int64_t msize, int64_t p, int nregs, int nzero,
-                          unsigned grid, cudaStream_t st) {
+                          int wmax, unsigned grid, cudaStream_t st) {
     const size_t staged = exec_staged_smem(msize, nregs);
-    if (staged && ensure_dyn_smem(reinterpret_cast<const void *>(exec_kernel<T, LAYOUT, true>), static_cast<int>(staged)))
-        launch(exec_kernel<T, LAYOUT, true>, grid, ex::kThreads, staged, st, pg, (long long)t, mem, (long long)msize,
-               (long long)p, nregs, nzero);
+    const size_t windowed = (static_cast<size_t>(nregs) * ex::kThreads + static_cast<size_t>(wmax) * ex::kPitch) * 4;
+    if (staged && ensure_dyn_smem(reinterpret_cast<const void *>(exec_kernel<T, LAYOUT, EX_STAGED>), static_cast<int>(staged)))
+        launch(exec_kernel<T, LAYOUT, EX_STAGED>, grid, ex::kThreads, staged, st, pg, (long long)t, mem,
+               (long long)msize, (long long)p, nregs, nzero);
+    else if (wmax > 0 && (BO_EX_WINDOW_COL || LAYOUT == BO_ROW_WISE) && ensure_dyn_smem(reinterpret_cast<const void *>(exec_kernel<T, LAYOUT, EX_WINDOWED>),
+                                         static_cast<int>(windowed)))
+        launch(exec_kernel<T, LAYOUT, EX_WINDOWED>, grid, ex::kThreads, windowed, st, pg, (long long)t, mem,
+               (long long)msize, (long long)p, nregs, nzero);
     else
-        launch(exec_kernel<T, LAYOUT, false>, grid, ex::kThreads, static_cast<size_t>(nregs) * ex::kThreads * 4, st, pg,
-               (long long)t, mem, (long long)msize, (long long)p, nregs, nzero);
+        launch(exec_kernel<T, LAYOUT, EX_DIRECT>, grid, ex::kThreads, static_cast<size_t>(nregs) * ex::kThreads * 4, st,
+               pg, (long long)t, mem, (long long)msize, (long long)p, nregs, nzero);
 }
 
 int launch_exec(const void *prog, int64_t t, void *mem, int64_t msize, int64_t p, int dtype, int layout, int nregs,
-                int nzero, cudaStream_t st) {
+                int nzero, int wmax, cudaStream_t st) {
     const unsigned grid = static_cast<unsigned>((p + ex::kThreads - 1) / ex::kThreads);
     const int4 *pg = static_cast<const int4 *>(prog);
     if (dtype == BO_F32) {
-        if (layout == BO_ROW_WISE) launch_exec_t<float, BO_ROW_WISE>(pg, t, static_cast<float *>(mem), msize, p, nregs, nzero, grid, st);
-        else launch_exec_t<float, BO_COLUMN_WISE>(pg, t, static_cast<float *>(mem), msize, p, nregs, nzero, grid, st);
+        if (layout == BO_ROW_WISE) launch_exec_t<float, BO_ROW_WISE>(pg, t, static_cast<float *>(mem), msize, p, nregs, nzero, wmax, grid, st);
+        else launch_exec_t<float, BO_COLUMN_WISE>(pg, t, static_cast<float *>(mem), msize, p, nregs, nzero, wmax, grid, st);
     } else {
-        if (layout == BO_ROW_WISE) launch_exec_t<int32_t, BO_ROW_WISE>(pg, t, static_cast<int32_t *>(mem), msize, p, nregs, nzero, grid, st);
-        else launch_exec_t<int32_t, BO_COLUMN_WISE>(pg, t, static_cast<int32_t *>(mem), msize, p, nregs, nzero, grid, st);
+        if (layout == BO_ROW_WISE) launch_exec_t<int32_t, BO_ROW_WISE>(pg, t, static_cast<int32_t *>(mem), msize, p, nregs, nzero, wmax, grid, st);
+        else launch_exec_t<int32_t, BO_COLUMN_WISE>(pg, t, static_cast<int32_t *>(mem), msize, p, nregs, nzero, wmax, grid, st);
     }
     return after_launch("exec_kernel");
 }

@@ -243,3 +243,44 @@ def test_prepared_program_in_captured_graph(layout):
         g.replay()
         torch.cuda.synchronize()
         assert np.array_equal(work.cpu().numpy(), ref)
+
+
+def _drifting_program(msize, nregs, t, seed):
+    """Random programs with locality: addresses drawn from a 40-word range that
+    drifts through the memory, so the executor cuts them into several shared-memory
+    windows (exec.cu, WIN) with registers, loads and stores crossing window changes."""
+    rng = np.random.default_rng(seed)
+    code, base = [], 0
+    r = lambda: int(rng.integers(0, nregs))
+    while len(code) < t:
+        base = min(base + int(rng.integers(0, 3)), msize - 40)
+        a = lambda: base + int(rng.integers(0, 40))
+        k = rng.random()
+        if k < 0.3:
+            A, B = (base + int(v) for v in rng.permutation(40)[:2])
+            code += [(0, 0, A, 0), (0, 1, B, 0), (4, 2, 0, 1), (5, 3, 0, 1), (1, A, 2, 0), (1, B, 3, 0)]
+        elif k < 0.5:
+            code += [(0, 4, a(), 0), (2, 5, 5, 4), (1, a(), 5, 0)]
+        else:
+            op = int(rng.choice([0, 1, 2, 3, 4, 5, 6]))
+            code.append((op, r(), a(), 0) if op == 0 else (op, a(), r(), 0) if op == 1 else (op, r(), r(), r()))
+    return np.asarray(code[:t], dtype=np.int32).reshape(-1, 4)
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("seed,t,msize,p", [(21, 3000, 500, 300), (22, 800, 200, 129), (23, 5000, 1000, 1000)])
+def test_executor_windowed_programs_match_oracle(dt, layout, seed, t, msize, p):
+    prog = _drifting_program(msize, 6, t, seed)
+    x = bulkgen.prefix_input(msize, p, seed=seed, dtype=dt, layout=layout)
+    ref = oracle.bulk_execute(prog, x, layout)
+    for run in ("call", "prepared"):
+        got = torch.from_numpy(x).to(DEV)
+        bo.execute(prog if run == "call" else bo.prepare(prog, msize), got, layout)
+        g = got.cpu().numpy()
+        r = ref
+        if dt == "float32":
+            nan = np.isnan(g)
+            assert np.array_equal(nan, np.isnan(r))
+            g, r = g[~nan], r[~nan]
+        assert np.array_equal(g.view(np.uint32), r.view(np.uint32)), run
