@@ -20,7 +20,10 @@
 //     group stores to takes the stored value), fetching the next word ahead;
 // (3) when the CTA's 128 instance memories fit (exec_staged_smem) they are
 //     staged in shared memory with coalesced copies, so every LOAD/STORE is a
-//     conflict-free shared access in either arrangement.
+//     conflict-free shared access in either arrangement; when they do not, a
+//     program with address locality is cut into windows (WIN words, see
+//     exec_device_program) and each window is staged the same way (row-wise
+//     only: column-wise accesses are already coalesced and measured faster).
 // The internal instructions:
 //   CE  = LOAD ra,A; LOAD rb,B; MIN rn,..; MAX rx,..; STORE S1,q1; STORE S2,q2
 //         (a compare-exchange: the whole bitonic network, programs.py), two
