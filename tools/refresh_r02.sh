@@ -23,6 +23,9 @@ prof tr2_tiled tri_tiled tri 64 65536 float32 0 20
 prof tr1_reg tri_thread_reg tri 16 65536 int32 0 18
 prof tr1col_reg tri_thread_reg tri 16 65536 int32 1 18
 prof ps32k_col ps_across prefix 32768 8192 float32 1 1
+prof exec_bitonic_col exec_kernel exec_bitonic 64 1048576 float32 1 0
+prof exec_prefix_col exec_kernel exec_prefix 1024 1048576 float32 1 0
+prof exec_prefix_row exec_kernel exec_prefix 1024 1048576 float32 0 0
 for tool in memcheck racecheck synccheck; do
   timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize.py > $OUT/sanitizer_$tool.log 2>&1
   echo "sanitizer $tool rc=$?"
