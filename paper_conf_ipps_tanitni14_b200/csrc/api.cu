@@ -266,7 +266,8 @@ static HostPipe *host_pipe() {
 }
 
 #ifndef BO_HOST_CHUNKS
-#define BO_HOST_CHUNKS 32     // measured: 8 -> 95.2 ms, 32 -> 89.8 ms per 8 GiB round trip (PCIe-bound)
+#define BO_HOST_CHUNKS 64     // measured: 8 -> 95.2 ms, 32 -> 89.8 ms per 8 GiB round trip (PCIe-bound);
+                              // r02 A/B on one box: 16 / 32 / 64 / 128 -> 96.5 / 94.0 / 91.4 / 93.3 ms
 #endif
 static int64_t host_chunk(int64_t p) {
     // BO_HOST_CHUNKS chunks, multiple of 128 instances, so copies of chunk k+1
