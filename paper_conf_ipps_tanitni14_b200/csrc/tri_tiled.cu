@@ -480,7 +480,86 @@ __device__ __forceinline__ void preload_table(T *Z, const T *__restrict__ c, lon
     }
 }
 
-template <typename T, int LPI, bool CHORDS>
+// Step 1 for a whole CTA batch of column-wise weights, whole sectors:
+// the CTA's ninst = 8 * groups instances are consecutive and 32-byte aligned,
+// so one 256-bit load brings cell (a, b) of 8 of them, and the thread writes
+// the 8 values into the 8 tables (one STS each).  Warp w takes the row pairs
+// (r, n-3-r), r = w, w + W, ... (n-1 cells per pair) in 32-cell pieces, so a
+// warp's lanes take consecutive cells of one row: 32 consecutive b of row a
+// land in distinct 16-byte bank groups (colbase(m) mod 8 runs through every
+// residue over 8 consecutive m).  The per-warp path above reads 8 of every 32
+// bytes it fetches and writes shared memory once per returning sector (ncu:
+// ~13 wavefronts per LDGSTS, L1 at 83 %); here a 32-byte sector is one lane's
+// load.  Called between two __syncthreads (the tables belong to all warps of
+// the CTA here).  R loads per lane in flight: R = 1 keeps the kernel at its
+// DP register count (148 at fp32 / 16 lanes); R = 2 / 4 (165 / 199 registers)
+// and 4-byte cp.async copies of every cell at once measured no faster (§11).
+template <typename T, int R = 1>
+__device__ __forceinline__ void coop_preload_column(T *Zcta, int words, const T *__restrict__ c, long long h0,
+                                                    int n, long long p, int layout, int groups) {
+    struct __align__(32) V8 { T v[8]; };
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+    const int npairs = (n - 1) >> 1;
+    // a warp's items: its row pairs r = warp, warp + nw, ... x 32-cell pieces k x sector groups g
+    const int lg = groups == 2 ? 1 : 0, lkp = n - 1 > 32 ? 1 : 0;   // (tiled kernels: n <= 64)
+    const int lpp = lg + lkp;
+    const int items = warp < npairs ? ((npairs - 1 - warp) / nw + 1) << lpp : 0;
+    for (int i0 = 0; i0 < items; i0 += R) {
+        V8 v[R];
+        int off[R], grp[R];
+        bool ok[R];
+#pragma unroll
+        for (int u = 0; u < R; ++u) {
+            const int it = i0 + u;
+            const int r = warp + nw * (it >> lpp), k = (it >> lg) & lkp, g = it & lg;
+            const int j = 32 * k + lane, L1 = n - 2 - r;
+            const int a = j < L1 ? r : n - 3 - r;
+            const int b = j < L1 ? r + 2 + j : a + 2 + (j - L1);
+            ok[u] = it < items && j < n - 1 && (j < L1 || a != r);
+            const long long e = layout == BO_COLUMN_WISE
+                                    ? static_cast<long long>(a) * n + b
+                                    : static_cast<long long>(a) * (n - 2) - static_cast<long long>(a) * (a - 1) / 2 + (b - a - 2);
+            off[u] = tt::xoff(a, b);
+            grp[u] = 8 * g;
+            if (ok[u]) v[u] = *reinterpret_cast<const V8 *>(c + e * p + h0 + 8 * g);
+        }
+#pragma unroll
+        for (int u = 0; u < R; ++u)
+            if (ok[u]) {
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const int t = grp[u] + i;                          // table (instance) of the CTA
+                    Zcta[t * words + off[u]] = v[u].v[i];
+                }
+            }
+    }
+}
+
+// Bulk L2 prefetch of the NEXT wave of column-wise weights.  The CTAs of one
+// wave (batch j of every CTA) cover the consecutive instances [w0, w0 +
+// inst_stride), so each weight row (a, b) of the wave is one contiguous run of
+// inst_stride * 4 bytes (14 KB for 444 CTAs x 8).  CTA k prefetches the runs of
+// cells e = k, k + gridDim.x, ... with cp.async.bulk.prefetch.L2, so DRAM
+// serves long sequential reads; the CTAs' own 32-byte loads then hit L2
+// (without it each CTA's 32-byte sectors, 4 p bytes apart, come from a
+// different DRAM row: ~2 TB/s for the copy phase alone).
+template <typename T>
+__device__ __forceinline__ void coop_bulk_prefetch_wave(const T *__restrict__ c, long long w0, long long span, int n,
+                                                        long long p, int layout) {
+    const int lane = threadIdx.x & 31;
+    if ((threadIdx.x >> 5) != 0 || w0 >= p) return;
+    const long long cnt = min(span, p - w0);
+    const unsigned bytes = static_cast<unsigned>(cnt * sizeof(T)) & ~15u;
+    if (bytes == 0) return;
+    const int cells = layout == BO_COLUMN_WISE ? n * n : (n - 1) * (n - 2) / 2;
+    for (int e = blockIdx.x + gridDim.x * lane; e < cells; e += 32 * gridDim.x) {
+        if (layout == BO_COLUMN_WISE && (e % n) < (e / n) + 2) continue;   // not read by Algorithm OPT
+        const T *src = c + static_cast<long long>(e) * p + w0;
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+    }
+}
+
+template <typename T, int LPI, bool CHORDS, bool COOP>
 __global__ void __launch_bounds__(128, 1)
 tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restrict__ chords, int n, long long p,
                  int layout, int NT, int c_vec, uint64_t lsched) {
@@ -498,6 +577,7 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
     const int slot = lane & (IPW - 1), li = lane >> kLogIpw;
     const int words = table_stride(NT, IPW);             // per-instance table size (+ bank pad)
     const int warps_per_cta = blockDim.x >> 5;
+    const int ninst = warps_per_cta * IPW;              // consecutive instances per CTA pass
     T *Z = reinterpret_cast<T *>(smem_raw) + static_cast<size_t>(warp * IPW + slot) * words;
 
     // zero the table once: padding cells then stay finite forever
@@ -507,7 +587,6 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
     const long long inst_stride = static_cast<long long>(gridDim.x) * warps_per_cta * IPW;
     const long long nn = static_cast<long long>(n) * n;
 
-    const int ninst = warps_per_cta * IPW;              // consecutive instances per CTA pass
     for (long long base = static_cast<long long>(blockIdx.x) * ninst; base < p; base += inst_stride) {
         const long long h = base + warp * IPW + slot;
         const bool live = h < p;
@@ -516,11 +595,25 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
 #endif
         // ------------------------------------------------ 1. c -> upper table
 #ifndef BO_TT_NOPRELOAD
-        preload_table<T, LPI>(Z, c, h, live, n, p, layout, NT, c_vec, li);
+        if (COOP && base + ninst <= p) {                   // CTA-uniform
+            __syncthreads();                                // every table of the CTA is free
+            BO_CLK_MARK(150);
+            coop_preload_column<T>(reinterpret_cast<T *>(smem_raw), words, c, base, n, p, layout, ninst >> 3);
+            BO_CLK_MARK(151);
+            __syncthreads();
+            BO_CLK_MARK(152);
+            // the next wave's rows into L2 (0.492 -> 0.488 ms at TR-2 column-wise; a
+            // per-sector prefetch of this CTA's next batch measured the same)
+            coop_bulk_prefetch_wave<T>(c, base - static_cast<long long>(blockIdx.x) * ninst + inst_stride, inst_stride, n, p,
+                                       layout);
+        } else {
+            preload_table<T, LPI>(Z, c, h, live, n, p, layout, NT, c_vec, li);
+        }
 #endif   // (-DBO_TT_NOPRELOAD: timing experiment only -- results are wrong)
         __syncwarp();
         BO_CLK_MARK(0);
 
+#ifndef BO_TT_COPYONLY   // (timing experiment: preload only, results are wrong)
         // ------------------------------------------------ 2. D = 0 (diagonal tiles)
         T dg0[3] = {T(0), T(0), T(0)}, dg1[3] = {T(0), T(0), T(0)};   // diag tiles li, li + LPI (upper part)
 #pragma unroll
@@ -594,6 +687,7 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             __syncwarp();
             BO_CLK_MARK(83 + 4 * D);
         }
+#endif   // BO_TT_COPYONLY
         if (live && li == 0) out[h] = Z[tt::xoff(0, n - 1)];   // X[0][n-1] = Algorithm OPT's M[1,n-1]
 
         if constexpr (CHORDS) {
@@ -680,6 +774,7 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
     const int NT = static_cast<int>((n + 3) / 4);
     constexpr int IPW = 32 / LPI;
     const size_t per_inst = static_cast<size_t>(table_stride(NT, IPW)) * sizeof(T);
+    const bool column = layout == BO_COLUMN_WISE || layout == BO_PACKED_COLUMN;
     // warps per CTA: the W in 1..4 that keeps the most warps resident per SM
     // (shared memory is the limit: 227 KB, 1 KB reserved per CTA)
     int W = 1, best = 0;
@@ -687,19 +782,26 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
         const size_t per_cta = w * IPW * per_inst + 1024;
         const int resident = static_cast<int>((227 * 1024) / per_cta) * w;
         // column-wise weights: prefer 4 warps (8+ consecutive instances = whole sectors)
-        if (resident > best || (layout == BO_COLUMN_WISE && resident == best)) best = resident, W = w;
+        if (resident > best || (column && resident == best)) best = resident, W = w;
     }
     const size_t smem = W * IPW * per_inst;
-    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(&tri_tiled_kernel<T, LPI, CHORDS>), 227 * 1024);
-    if (!attr) return fail(BO_ECUDA, "tiled: cannot set dynamic smem");
-    int per_sm = 1;
-    per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(&tri_tiled_kernel<T, LPI, CHORDS>), W * 32, smem);
-    per_sm = std::max(per_sm, 1);
     const long long per_cta = static_cast<long long>(W) * IPW;
+    const int c_vec = (n % 4 == 0) && aligned16(c);
+    // whole-sector CTA preload of column-wise weights (8 or 16 consecutive,
+    // 32-byte aligned instances per CTA batch): a kernel of its own, so the
+    // per-warp kernels keep their register allocation
+    bool coop = false;
+#ifndef BO_TT_NOCOOP
+    coop = column && (per_cta == 8 || per_cta == 16) && p % 8 == 0 && (reinterpret_cast<uintptr_t>(c) & 31u) == 0;
+#endif
+    const auto kern = coop ? &tri_tiled_kernel<T, LPI, CHORDS, true> : &tri_tiled_kernel<T, LPI, CHORDS, false>;
+    const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(kern), 227 * 1024);
+    if (!attr) return fail(BO_ECUDA, "tiled: cannot set dynamic smem");
+    int per_sm = max_blocks_per_sm(reinterpret_cast<const void *>(kern), W * 32, smem);
+    per_sm = std::max(per_sm, 1);
     const long long blocks = std::min<long long>((p + per_cta - 1) / per_cta,
                                                  static_cast<long long>(per_sm) * num_sms());
-    const int c_vec = (n % 4 == 0) && aligned16(c);
-    launch(tri_tiled_kernel<T, LPI, CHORDS>, static_cast<unsigned>(blocks), W * 32, smem, st, 
+    launch(kern, static_cast<unsigned>(blocks), W * 32, smem, st,
         static_cast<const T *>(c), static_cast<T *>(out), chords, static_cast<int>(n), p, layout, NT, c_vec,
         split_schedule(NT, LPI));
     return after_launch("tri_tiled_kernel");

@@ -309,3 +309,29 @@ def test_full_inputs_tr1_tr2_shapes(layout):
         ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 24, dt, kind="full"), oracle.ROW_WISE,
                               nthreads=NTHREADS)
         assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32)), (n, layout)
+
+
+# Column-wise weights through the CTA-cooperative whole-sector preload (tiled kernels with
+# 8 or 16 consecutive instances per CTA batch, p % 8 == 0, 32-byte aligned weights):
+# every CTA runs several batches, p % 16 == 8 leaves a per-warp tail batch for the
+# 16-instance CTAs, and an offset view (not 32-byte aligned) takes the per-warp path.
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.COLUMN_WISE, bo.PACKED_COLUMN])
+@pytest.mark.parametrize("n,p", [(5, 40008), (8, 24000), (13, 16008), (17, 12000), (24, 9992), (33, 8008),
+                                 (40, 6000), (61, 4008), (63, 4000), (64, 12008)])
+def test_coop_column_preload_full_inputs(dt, layout, n, p):
+    c = bulkgen.tri_input(n, p, seed=31 * n + p, dtype=dt, layout=layout, kind="full")
+    ids = np.unique(np.r_[np.arange(0, p, 5), np.arange(p - 24, p)])
+    ct = torch.from_numpy(c).to(DEV)
+    ref = oracle.bulk_opt(bulkgen.tri_instances(n, ids, 31 * n + p, dt, kind="full"), oracle.ROW_WISE,
+                          nthreads=NTHREADS)
+    for v in [bo.AUTO, bo.TRI_TILED, bo.TRI_TILED_HALF, bo.TRI_TILED_QUARTER]:
+        if _supported(n, v):
+            got = bo.triangulation(ct, layout, v).cpu().numpy()
+            assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32)), (n, v)
+    # the same weights 4 bytes off a 32-byte boundary (per-warp preload path)
+    buf = torch.empty(ct.numel() + 8, dtype=ct.dtype, device=DEV)
+    off = buf[1:1 + ct.numel()].view(ct.shape)
+    off.copy_(ct)
+    got = bo.triangulation(off, layout, bo.TRI_TILED_HALF if n <= 64 else bo.AUTO).cpu().numpy()
+    assert np.array_equal(got[ids].view(np.uint32), ref.view(np.uint32)), n
