@@ -28,6 +28,10 @@ for layout in (bo.PACKED_ROW, bo.PACKED_COLUMN):
         c = bo.generate_tri(n, p, 1, torch.float32, layout)
         bo.triangulation(c, layout)
         bo.triangulation_chords(c, layout)
+# the CTA-cooperative column-wise preload over several batches per CTA (+ a per-warp tail batch)
+for layout in (bo.COLUMN_WISE, bo.PACKED_COLUMN):
+    for n, p, v in ((16, 7112, bo.TRI_TILED_HALF), (24, 7112, bo.TRI_TILED_QUARTER)):
+        bo.triangulation(bo.generate_tri(n, p, 1, torch.float32, layout), layout, v)
 c = bo.generate_tri(80, 3, 1, torch.float32, bo.ROW_WISE)
 bo.triangulation(c, bo.ROW_WISE, bo.TRI_TILED_GLOBAL)
 bo.triangulation(c, bo.ROW_WISE, bo.TRI_TILED_GLOBAL8)
