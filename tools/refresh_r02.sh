@@ -1,6 +1,6 @@
 #!/bin/bash
 # Round-2 evidence refresh on the GPU box (gpurun): full -m gpu suite, smoke, bench line, the ncu
-# launch list of the bench command, one `ncu --set full` capture per hot kernel, sanitizers.
+# launch list of the bench command, one `ncu --set full` capture per hot kernel, the p-sweep.
 # Outputs in gpurun_out/; summaries go to profiles/r02/ (tools/ncu_summarize.py, run locally).
 set -u
 OUT=gpurun_out
@@ -23,11 +23,11 @@ prof tr2_tiled tri_tiled tri 64 65536 float32 0 20
 prof tr1_reg tri_thread_reg tri 16 65536 int32 0 18
 prof tr1col_reg tri_thread_reg tri 16 65536 int32 1 18
 prof ps32k_col ps_across prefix 32768 8192 float32 1 1
+prof tr2col_tiled tri_tiled tri 64 65536 float32 1 0
+prof tr2pcol_tiled tri_tiled tri 64 65536 float32 3 0
 prof exec_bitonic_col exec_kernel exec_bitonic 64 1048576 float32 1 0
 prof exec_prefix_col exec_kernel exec_prefix 1024 1048576 float32 1 0
 prof exec_prefix_row exec_kernel exec_prefix 1024 1048576 float32 0 0
-for tool in memcheck racecheck synccheck; do
-  timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize.py > $OUT/sanitizer_$tool.log 2>&1
-  echo "sanitizer $tool rc=$?"
-done
+# (compute-sanitizer was closed on the GPU pool late in round 2; the r02 sanitizer logs predate the
+#  cooperative column-wise preload)
 timeout 1200 python bench.py --sweep > $OUT/sweep.json 2> $OUT/sweep.err; echo "sweep rc=$?"
