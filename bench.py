@@ -88,6 +88,15 @@ WORKLOADS = {
                             variant=0, desc="NEXT-3: generic executor running Algorithm Prefix-sums, column-wise"),
     "exec_prefix_row": dict(seed=2, algo="exec", prog="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0,
                             variant=0, desc="NEXT-3: generic executor running Algorithm Prefix-sums, row-wise, windowed in shared memory"),
+    "exec_bitonic_col_jit": dict(seed=6, algo="exec", prog="bitonic", n=64, p=2 ** 20, dtype="float32", layout=1,
+                                 variant=0, jit=True,
+                                 desc="NEXT-3: the bitonic sort program compiled to a straight-line kernel (bulk_program_compile), column-wise"),
+    "exec_bitonic_row_jit": dict(seed=6, algo="exec", prog="bitonic", n=64, p=2 ** 20, dtype="float32", layout=0,
+                                 variant=0, jit=True,
+                                 desc="NEXT-3: the bitonic sort program compiled, row-wise (rows staged in shared memory)"),
+    "exec_prefix_col_jit": dict(seed=2, algo="exec", prog="prefix", n=1024, p=2 ** 20, dtype="float32", layout=1,
+                                variant=0, jit=True,
+                                desc="NEXT-3: Algorithm Prefix-sums as a program, compiled (streaming shape), column-wise"),
     # the paper's other experiment shapes (§V): n = 32K floats at p = 8K, 8-gons at
     # p = 4M, our kernels beside the paper's naive row-/column-wise kernels (Figs. 11, 12)
     "ps32k": dict(seed=21, algo="prefix", n=32768, p=8192, dtype="float32", layout=0, variant=0,
@@ -111,6 +120,7 @@ WORKLOADS = {
 }
 EXTRAS = ["ps2col", "ps2tr", "tr_transpose", "ps1", "tr1", "tr1col", "tr1packed", "tr2", "tr2col", "tr2packed", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
           "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col", "exec_prefix_row",
+          "exec_bitonic_col_jit", "exec_bitonic_row_jit", "exec_prefix_col_jit",
           "ps32k", "ps32k_col", "ps32k_naive_row", "ps32k_naive_col", "tr8", "tr8col", "tr8_umm_row", "tr8_umm_col"]
 # The paper's own fitted GTX Titan models, in ms for p instances: context for the
 # extras of the same shape, never a target (another machine, another decade)
@@ -347,12 +357,15 @@ def setup_workload(wl, rank, copies=1):
         prog = programs.bitonic_sort(n) if wl["prog"] == "bitonic" else programs.prefix_sums(n, wl["dtype"])
         x = bo.generate_prefix(n, p, seed, dt, wl["layout"], "uniform", h0=h0)
         prep = bo.prepare(prog, n)          # validated, rewritten and uploaded once, outside the timed steps
+        how = "prepared"
+        if wl.get("jit"):                   # NVRTC-compiled straight-line kernel, built outside the timed steps
+            how = "compiled" if prep.compile(dt, wl["layout"]) else "prepared (not compiled)"
         nxt = _rotator(x, copies)
 
         def fn():
             bo.execute(prep, nxt(), wl["layout"])
         return dict(x=x, out=x, fn=fn, seed=seed, h0=h0, prep=prep,
-                    variant=f"exec[{wl['prog']}: {prog.array().shape[0]} instr, prepared]")
+                    variant=f"exec[{wl['prog']}: {prog.array().shape[0]} instr, {how}]")
     if wl["algo"] == "transpose":
         x = bo.generate_prefix(n, p, seed, dt, bo.ROW_WISE, "uniform", h0=h0)        # [p][n]
         out = torch.empty((n, p), dtype=dt, device="cuda")

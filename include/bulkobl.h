@@ -204,6 +204,31 @@ int bulk_execute_prepared(int64_t handle, void *mem, int64_t msize, int64_t p, i
 int bulk_program_release(int64_t handle);
 
 /* ------------------------------------------------------------------------- */
+/* Compiled programs (NEXT-3).  Obliviousness makes every address of a */
+/* program a constant, so the bulk execution of Theorem 2 can be  */
+/* one straight-line kernel: the program unrolled, the instance memory in     */
+/* registers.  The paper leaves a converter from sequential code to its bulk  */
+/* CUDA program as future work; this compiles the IR above.           */
+/*   bulk_program_compile: builds, with NVRTC for sm_100a (host-blocking,     */
+/*     ~0.1-2 s; cached process-wide by the generated source), the kernel of  */
+/*     the prepared program `handle` for one dtype and layout; afterwards     */
+/*     bulk_execute_prepared with that dtype and layout launches it instead   */
+/*     of the interpreter (same results bit for bit; still capturable).       */
+/*     Shapes: column-wise any msize (msize <= 128: memory in registers,      */
+/*     coalesced load / store of the words read / written; larger: direct     */
+/*     loads grouped 16 at a time); row-wise msize <= 95 (rows staged through  */
+/*     shared memory).  BO_EUNSUPPORTED otherwise (row-wise msize > 95, more  */
+/*     than 200000 instructions) -- the interpreter keeps serving the call;   */
+/*     BO_ECUDA with the NVRTC log if compilation fails; BO_EINVAL on an      */
+/*     unknown handle or a packed layout.  Not while a stream is capturing.   */
+/*   bulk_program_source: the CUDA source bulk_program_compile builds (NUL-   */
+/*     terminated); *len = bytes needed incl. the NUL; copied only when       */
+/*     cap >= *len.                                                           */
+/* ------------------------------------------------------------------------- */
+int bulk_program_compile(int64_t handle, int dtype, int layout);
+int bulk_program_source(int64_t handle, int dtype, int layout, char *buf, size_t cap, size_t *len);
+
+/* ------------------------------------------------------------------------- */
 /* Layout transpose (row-wise <-> column-wise arrangement):        */
 /*   dst[c*rows + r] = src[r*cols + c],  0 <= r < rows, 0 <= c < cols.        */
 /* Row-wise [p][n] -> column-wise [n][p] is (rows=p, cols=n); the reverse is  */

@@ -67,6 +67,8 @@ def lib() -> ctypes.CDLL:
             "bulk_execute": ([vp, i64, vp, sz, vp, i64, i64, i32, i32, i32, vp], i32),
             "bulk_program_prepare": ([vp, i64, i64, i32, vp, sz, vp, ctypes.POINTER(i64)], i32),
             "bulk_execute_prepared": ([i64, vp, i64, i64, i32, i32, vp], i32),
+            "bulk_program_compile": ([i64, i32, i32], i32),
+            "bulk_program_source": ([i64, i32, i32, vp, sz, ctypes.POINTER(sz)], i32),
             "bulk_program_release": ([i64], i32),
             "bulk_prefix_sums_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_triangulation_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
@@ -92,6 +94,9 @@ def lib() -> ctypes.CDLL:
 def _check(rc: int):
     if rc != 0:
         raise BulkError(rc, lib().bulk_last_error().decode())
+
+
+_DTYPES = {torch.int32: 0, torch.float32: 1, "int32": 0, "float32": 1}
 
 
 def _dtype_code(t: torch.Tensor) -> int:
@@ -298,6 +303,28 @@ class Prepared:
         _check(lib().bulk_program_prepare(code.ctypes.data, self.t, self.msize, self.nregs, self.buf.data_ptr(),
                                           self.buf.numel(), _stream(stream, self.buf), ctypes.byref(h)))
         self.handle = h.value
+
+    def compile(self, dtype=torch.float32, layout: int = COLUMN_WISE) -> bool:
+        """Build the straight-line kernel of this program for (dtype, layout)
+        (bulk_program_compile, NVRTC for sm_100a; host-blocking, cached).  True
+        when later execute() calls with that dtype and layout run it; False when
+        the shape is not compiled (row-wise with msize > 95) and the
+        interpreter keeps serving them."""
+        code = _DTYPES[dtype] if not isinstance(dtype, int) else dtype
+        rc = lib().bulk_program_compile(self.handle, code, layout)
+        if rc == -2:
+            return False
+        _check(rc)
+        return True
+
+    def source(self, dtype=torch.float32, layout: int = COLUMN_WISE) -> str:
+        """The CUDA source compile() builds for (dtype, layout)."""
+        code = _DTYPES[dtype] if not isinstance(dtype, int) else dtype
+        n = ctypes.c_size_t(0)
+        _check(lib().bulk_program_source(self.handle, code, layout, None, 0, ctypes.byref(n)))
+        buf = ctypes.create_string_buffer(n.value)
+        _check(lib().bulk_program_source(self.handle, code, layout, buf, n.value, ctypes.byref(n)))
+        return buf.value.decode()
 
     def __del__(self):
         if getattr(self, "handle", 0) and _lib is not None:

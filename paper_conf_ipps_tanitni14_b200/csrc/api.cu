@@ -3,6 +3,7 @@
 // host-buffer entry points.  No computation happens on the CPU.
 #include "common.cuh"
 #include "exec.h"
+#include "jit.h"
 
 #include <cstring>
 #include <mutex>
@@ -414,9 +415,11 @@ struct PreparedProgram {
     const void *dev;
     int64_t tu, msize;
     int nregs, nzero, wmax;
+    const void *jit[2][2];      // compiled kernels [dtype][layout] (bulk_program_compile), or null
 };
 std::mutex g_prep_mu;
 std::map<int64_t, PreparedProgram> g_prep;
+std::map<int64_t, std::vector<int32_t>> g_prep_src;   // the validated program as given (for compiling)
 int64_t g_prep_next = 1;
 }  // namespace
 
@@ -448,7 +451,8 @@ int bulk_program_prepare(const int32_t *prog, int64_t t, int64_t msize, int nreg
     }
     std::lock_guard<std::mutex> g(g_prep_mu);
     const int64_t h = g_prep_next++;
-    g_prep[h] = PreparedProgram{prog_dev, tu, msize, nregs, uninit_read ? nregs : 0, ep.wmax};
+    g_prep[h] = PreparedProgram{prog_dev, tu, msize, nregs, uninit_read ? nregs : 0, ep.wmax, {{nullptr, nullptr}, {nullptr, nullptr}}};
+    g_prep_src[h].assign(prog, prog + 4 * t);
     *handle = h;
     return BO_OK;
 }
@@ -467,6 +471,8 @@ int bulk_execute_prepared(int64_t handle, void *mem, int64_t msize, int64_t p, i
     if (!valid_dtype(dtype) || !valid_layout(layout)) return fail(BO_EINVAL, "execute: bad dtype or layout");
     if (pp.tu == 0 || p == 0) return BO_OK;
     if (!mem) return fail(BO_EINVAL, "execute: NULL pointer");
+    if ((layout == BO_ROW_WISE || layout == BO_COLUMN_WISE) && pp.jit[dtype][layout])
+        return launch_jit(JitKernel{pp.jit[dtype][layout]}, mem, p, static_cast<cudaStream_t>(stream));
     return launch_exec(pp.dev, pp.tu, mem, msize, p, dtype, layout, pp.nregs, pp.nzero, pp.wmax,
                        static_cast<cudaStream_t>(stream));
 }
@@ -475,6 +481,51 @@ int bulk_program_release(int64_t handle) {
     t_err.clear();
     std::lock_guard<std::mutex> g(g_prep_mu);
     if (g_prep.erase(handle) == 0) return fail(BO_EINVAL, "release: unknown program handle");
+    g_prep_src.erase(handle);
+    return BO_OK;
+}
+
+int bulk_program_compile(int64_t handle, int dtype, int layout) {
+    t_err.clear();
+    if (!valid_dtype(dtype) || (layout != BO_ROW_WISE && layout != BO_COLUMN_WISE))
+        return fail(BO_EINVAL, "compile: dtype BO_I32 / BO_F32, layout BO_ROW_WISE / BO_COLUMN_WISE");
+    std::vector<int32_t> src;
+    PreparedProgram pp;
+    {
+        std::lock_guard<std::mutex> g(g_prep_mu);
+        auto it = g_prep.find(handle);
+        if (it == g_prep.end()) return fail(BO_EINVAL, "compile: unknown program handle");
+        pp = it->second;
+        src = g_prep_src[handle];
+    }
+    if (pp.jit[dtype][layout]) return BO_OK;
+    JitKernel k;
+    const int64_t t = static_cast<int64_t>(src.size() / 4);
+    if (int rc = jit_compile(src.data(), t, pp.msize, pp.nregs, dtype, layout, &k)) return rc;
+    std::lock_guard<std::mutex> g(g_prep_mu);
+    auto it = g_prep.find(handle);
+    if (it == g_prep.end()) return fail(BO_EINVAL, "compile: program released while compiling");
+    it->second.jit[dtype][layout] = k.kernel;
+    return BO_OK;
+}
+
+int bulk_program_source(int64_t handle, int dtype, int layout, char *buf, size_t cap, size_t *len) {
+    t_err.clear();
+    if (!len) return fail(BO_EINVAL, "program source: NULL len");
+    std::vector<int32_t> src;
+    PreparedProgram pp;
+    {
+        std::lock_guard<std::mutex> g(g_prep_mu);
+        auto it = g_prep.find(handle);
+        if (it == g_prep.end()) return fail(BO_EINVAL, "program source: unknown program handle");
+        pp = it->second;
+        src = g_prep_src[handle];
+    }
+    if (!valid_dtype(dtype)) return fail(BO_EINVAL, "program source: bad dtype");
+    const std::string s = jit_source(src.data(), static_cast<int64_t>(src.size() / 4), pp.msize, pp.nregs, dtype, layout);
+    if (s.empty()) return fail(BO_EUNSUPPORTED, "program source: this arrangement is not compiled");
+    *len = s.size() + 1;
+    if (buf && cap >= s.size() + 1) std::memcpy(buf, s.c_str(), s.size() + 1);
     return BO_OK;
 }
 

@@ -480,7 +480,8 @@ __device__ __forceinline__ void preload_table(T *Z, const T *__restrict__ c, lon
     }
 }
 
-// Step 1 for a whole CTA batch of column-wise weights, whole sectors:
+// Step 1 for a whole CTA batch of column-wise weights, whole sectors
+// (and of packed row-wise weights, below):
 // the CTA's ninst = 8 * groups instances are consecutive and 32-byte aligned,
 // so one 256-bit load brings cell (a, b) of 8 of them, and the thread writes
 // the 8 values into the 8 tables (one STS each).  Warp w takes the row pairs
@@ -516,12 +517,24 @@ __device__ __forceinline__ void coop_preload_column(T *Zcta, int words, const T 
             const int a = j < L1 ? r : n - 3 - r;
             const int b = j < L1 ? r + 2 + j : a + 2 + (j - L1);
             ok[u] = it < items && j < n - 1 && (j < L1 || a != r);
-            const long long e = layout == BO_COLUMN_WISE
-                                    ? static_cast<long long>(a) * n + b
-                                    : static_cast<long long>(a) * (n - 2) - static_cast<long long>(a) * (a - 1) / 2 + (b - a - 2);
+            const bool dense = layout == BO_COLUMN_WISE || layout == BO_ROW_WISE;
+            const long long e = dense ? static_cast<long long>(a) * n + b
+                                      : static_cast<long long>(a) * (n - 2) - static_cast<long long>(a) * (a - 1) / 2 + (b - a - 2);
             off[u] = tt::xoff(a, b);
             grp[u] = 8 * g;
-            if (ok[u]) v[u] = *reinterpret_cast<const V8 *>(c + e * p + h0 + 8 * g);
+            if (ok[u]) {
+                if (layout == BO_COLUMN_WISE || layout == BO_PACKED_COLUMN) {
+                    v[u] = *reinterpret_cast<const V8 *>(c + e * p + h0 + 8 * g);
+                } else {
+                    // row-wise / packed row-wise: instance h's weights are one contiguous
+                    // row of `rs` words, so the warp's 32 consecutive cells of one
+                    // instance are one coalesced 128-byte request
+                    const long long rs = dense ? static_cast<long long>(n) * n : static_cast<long long>(n - 1) * (n - 2) / 2;
+                    const T *src = c + (h0 + 8 * g) * rs + e;
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) v[u].v[i] = src[i * rs];
+                }
+            }
         }
 #pragma unroll
         for (int u = 0; u < R; ++u)
@@ -604,8 +617,9 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
             BO_CLK_MARK(152);
             // the next wave's rows into L2 (0.492 -> 0.488 ms at TR-2 column-wise; a
             // per-sector prefetch of this CTA's next batch measured the same)
-            coop_bulk_prefetch_wave<T>(c, base - static_cast<long long>(blockIdx.x) * ninst + inst_stride, inst_stride, n, p,
-                                       layout);
+            if (layout == BO_COLUMN_WISE || layout == BO_PACKED_COLUMN)
+                coop_bulk_prefetch_wave<T>(c, base - static_cast<long long>(blockIdx.x) * ninst + inst_stride, inst_stride, n,
+                                           p, layout);
         } else {
             preload_table<T, LPI>(Z, c, h, live, n, p, layout, NT, c_vec, li);
         }
@@ -781,8 +795,10 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
     for (int w = 1; w <= 4; ++w) {
         const size_t per_cta = w * IPW * per_inst + 1024;
         const int resident = static_cast<int>((227 * 1024) / per_cta) * w;
-        // column-wise weights: prefer 4 warps (8+ consecutive instances = whole sectors)
-        if (resident > best || (column && resident == best)) best = resident, W = w;
+        // (column-wise and packed row-wise weights: prefer 4 warps, 8+ instances per batch for the
+        // cooperative preload)
+        const bool prefer4 = column || layout == BO_PACKED_ROW;
+        if (resident > best || (prefer4 && resident == best)) best = resident, W = w;
     }
     const size_t smem = W * IPW * per_inst;
     const long long per_cta = static_cast<long long>(W) * IPW;
@@ -792,7 +808,10 @@ static int launch_tiled_t(const void *c, void *out, int16_t *chords, int64_t n, 
     // per-warp kernels keep their register allocation
     bool coop = false;
 #ifndef BO_TT_NOCOOP
-    coop = column && (per_cta == 8 || per_cta == 16) && p % 8 == 0 && (reinterpret_cast<uintptr_t>(c) & 31u) == 0;
+    // (packed row-wise too: scalar loads, no alignment needed -- TR-2 packed 0.620 -> 0.499 ms; dense
+    // row-wise stays per-warp: its 16-byte cp.async rows measured 0.371 against 0.512 ms cooperative)
+    coop = (column && p % 8 == 0 && (reinterpret_cast<uintptr_t>(c) & 31u) == 0) || layout == BO_PACKED_ROW;
+    coop = coop && (per_cta == 8 || per_cta == 16);
 #endif
     const auto kern = coop ? &tri_tiled_kernel<T, LPI, CHORDS, true> : &tri_tiled_kernel<T, LPI, CHORDS, false>;
     const bool attr = ensure_dyn_smem(reinterpret_cast<const void *>(kern), 227 * 1024);

@@ -284,3 +284,87 @@ def test_executor_windowed_programs_match_oracle(dt, layout, seed, t, msize, p):
             assert np.array_equal(nan, np.isnan(r))
             g, r = g[~nan], r[~nan]
         assert np.array_equal(g.view(np.uint32), r.view(np.uint32)), run
+
+
+# ---------------------------------------------------------------------------
+# Compiled programs (bulk_program_compile, jit.cu): the straight-line kernels
+# NVRTC builds from a prepared program, bit for bit against the oracle
+# interpreter -- registers in memory (column-wise msize <= 128, row-wise <= 95
+# through shared memory) and the streaming shape (column-wise, larger msize,
+# loads grouped ahead of their block with store-to-load forwarding).
+# ---------------------------------------------------------------------------
+def _compiled_case(kind, msize, t, seed, dt):
+    if kind == "random":
+        return _random_program(msize, 7, t, seed, dt)
+    if kind == "fusable":
+        return _fusable_program(msize, 6, t, seed)
+    if kind == "bitonic":
+        return programs.bitonic_sort(msize).array()
+    return programs.prefix_sums(msize, dt).array()
+
+
+@pytest.mark.parametrize("dt", ["int32", "float32"])
+@pytest.mark.parametrize("layout", [bo.ROW_WISE, bo.COLUMN_WISE])
+@pytest.mark.parametrize("kind,msize,t,seed", [("random", 8, 300, 21), ("random", 64, 2000, 22), ("random", 95, 1500, 23),
+                                               ("random", 96, 900, 24), ("random", 130, 1500, 25),
+                                               ("random", 400, 1500, 26), ("fusable", 9, 600, 27),
+                                               ("fusable", 300, 800, 28), ("bitonic", 64, 0, 0), ("bitonic", 1, 0, 0),
+                                               ("prefix", 33, 0, 0), ("prefix", 300, 0, 0)])
+def test_compiled_program_matches_oracle(dt, layout, kind, msize, t, seed):
+    prog = _compiled_case(kind, msize, t, seed, dt)
+    prep = bo.prepare(prog, msize)
+    compiled = prep.compile(getattr(torch, dt), layout)
+    assert compiled == (layout == bo.COLUMN_WISE or msize <= 95)
+    if compiled:
+        assert "bo_prog" in prep.source(getattr(torch, dt), layout)
+    for p in (301, 128, 1):
+        x = bulkgen.prefix_input(msize, p, seed=seed + p, dtype=dt, layout=layout)
+        if dt == "float32":
+            x = (x * 8).astype(np.float32)
+        ref = oracle.bulk_execute(prog, x, layout)
+        g = bo.execute(prep, torch.from_numpy(x).to(DEV), layout).cpu().numpy()
+        if dt == "float32":
+            nan = np.isnan(g)
+            assert np.array_equal(nan, np.isnan(ref))
+            g, ref = g[~nan], ref[~nan]
+        assert np.array_equal(g.view(np.uint32), ref.view(np.uint32)), (kind, msize, p)
+
+
+def test_compiled_program_nan_and_signed_zero_semantics():
+    # MIN / MAX are the header's comparisons, not fminf / fmaxf: with a NaN or -0.0 operand
+    # the compiled kernel must pick exactly the operand the interpreter picks
+    vals = np.array([np.nan, -0.0, 0.0, 1.0, -np.inf, np.inf, -1.0], dtype=np.float32)
+    prog = []
+    out = 0
+    for i in range(len(vals)):
+        for j in range(len(vals)):
+            prog += [(0, 0, i, 0), (0, 1, j, 0), (4, 2, 0, 1), (5, 3, 0, 1), (3, 4, 0, 1),
+                     (1, 7 + out, 2, 0), (1, 8 + out, 3, 0), (1, 9 + out, 4, 0)]
+            out += 3
+    prog = np.asarray(prog, dtype=np.int32)
+    msize = 7 + out
+    x = np.zeros((msize, 64), dtype=np.float32)
+    x[:7] = vals[:, None]
+    ref = oracle.bulk_execute(prog, x, bo.COLUMN_WISE)
+    prep = bo.prepare(prog, msize)
+    assert prep.compile(torch.float32, bo.COLUMN_WISE)
+    g = bo.execute(prep, torch.from_numpy(x).to(DEV), bo.COLUMN_WISE).cpu().numpy()
+    nan = np.isnan(ref)
+    assert np.array_equal(np.isnan(g), nan)
+    assert np.array_equal(g[~nan].view(np.uint32), ref[~nan].view(np.uint32))
+
+
+def test_compiled_program_in_captured_graph():
+    n, p = 64, 1000
+    P = programs.bitonic_sort(n)
+    prep = bo.prepare(P, n)
+    assert prep.compile(torch.int32, bo.COLUMN_WISE)
+    x = bulkgen.prefix_input(n, p, seed=5, dtype="int32", layout=bo.COLUMN_WISE)
+    ref = oracle.bulk_execute(P.array(), x, bo.COLUMN_WISE)
+    buf = torch.from_numpy(x).to(DEV)
+    work = buf.clone()
+    g = bo.Captured(lambda s: (work.copy_(buf), bo.execute(prep, work, bo.COLUMN_WISE, stream=s)))
+    for _ in range(2):
+        g.replay()
+    torch.cuda.synchronize()
+    assert np.array_equal(work.cpu().numpy(), ref)

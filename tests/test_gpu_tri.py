@@ -312,11 +312,12 @@ def test_full_inputs_tr1_tr2_shapes(layout):
 
 
 # Column-wise weights through the CTA-cooperative whole-sector preload (tiled kernels with
-# 8 or 16 consecutive instances per CTA batch, p % 8 == 0, 32-byte aligned weights):
+# 8 or 16 consecutive instances per CTA batch, p % 8 == 0, 32-byte aligned weights; packed
+# row-wise weights take the cooperative path at any p and alignment):
 # every CTA runs several batches, p % 16 == 8 leaves a per-warp tail batch for the
 # 16-instance CTAs, and an offset view (not 32-byte aligned) takes the per-warp path.
 @pytest.mark.parametrize("dt", ["int32", "float32"])
-@pytest.mark.parametrize("layout", [bo.COLUMN_WISE, bo.PACKED_COLUMN])
+@pytest.mark.parametrize("layout", [bo.COLUMN_WISE, bo.PACKED_COLUMN, bo.PACKED_ROW])
 @pytest.mark.parametrize("n,p", [(5, 40008), (8, 24000), (13, 16008), (17, 12000), (24, 9992), (33, 8008),
                                  (40, 6000), (61, 4008), (63, 4000), (64, 12008)])
 def test_coop_column_preload_full_inputs(dt, layout, n, p):
