@@ -216,7 +216,7 @@ int bulk_program_release(int64_t handle);
 /*     of the interpreter (same results bit for bit; still capturable).       */
 /*     Shapes: column-wise any msize (msize <= 128: memory in registers,      */
 /*     coalesced load / store of the words read / written; larger: direct     */
-/*     loads grouped 16 at a time); row-wise msize <= 95 (rows staged through  */
+/*     loads grouped 32 at a time); row-wise msize <= 95 (rows staged through  */
 /*     shared memory).  BO_EUNSUPPORTED otherwise (row-wise msize > 95, more  */
 /*     than 200000 instructions) -- the interpreter keeps serving the call;   */
 /*     BO_ECUDA with the NVRTC log if compilation fails; BO_EINVAL on an      */
