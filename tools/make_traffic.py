@@ -13,7 +13,9 @@ import sys
 MAP = {"ps2": "ps2_fused", "ps2col": "ps2_across", "tr2": "tr2_tiled", "tr1": "tr1_reg", "tr_transpose": "transpose",
        "tr1col": "tr1col_reg", "tr2col": "tr2col_tiled", "tr2chords": "chords", "ps32k": "ps32k_row",
        "ps32k_col": "ps32k_col", "exec_bitonic_col": "exec_bitonic_col", "exec_prefix_col": "exec_prefix_col",
-       "exec_prefix_row": "exec_prefix_row"}
+       "exec_prefix_row": "exec_prefix_row",
+       "exec_bitonic_col_jit": "exec_bitonic_col_jit", "exec_bitonic_row_jit": "exec_bitonic_row_jit",
+       "exec_prefix_col_jit": "exec_prefix_col_jit", "tr2packed": "tr2prow_tiled"}
 
 
 def main():

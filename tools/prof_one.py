@@ -1,6 +1,7 @@
 #!/usr/bin/env python
 """Run one op a few times (for ncu).
-    python tools/prof_one.py prefix|tri|transpose|exec_prefix|exec_bitonic n p dtype layout variant [reps]"""
+    python tools/prof_one.py prefix|tri|transpose|exec_prefix|exec_bitonic n p dtype layout variant [reps]
+(exec_*: variant 1 = compiled program)"""
 import os
 import sys
 
@@ -32,6 +33,9 @@ elif algo.startswith("exec_"):
     from paper_conf_ipps_tanitni14_b200 import programs
     P = programs.prefix_sums(n, sys.argv[4]) if algo == "exec_prefix" else programs.bitonic_sort(n)
     x = bo.generate_prefix(n, p, 2, dt, layout)
+    if variant == 1:                       # variant 1: the compiled program (bulk_program_compile)
+        P = bo.prepare(P, n)
+        assert P.compile(dt, layout)
     for _ in range(reps):
         bo.execute(P, x, layout)
 else:

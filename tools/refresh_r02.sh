@@ -25,9 +25,13 @@ prof tr1col_reg tri_thread_reg tri 16 65536 int32 1 18
 prof ps32k_col ps_across prefix 32768 8192 float32 1 1
 prof tr2col_tiled tri_tiled tri 64 65536 float32 1 0
 prof tr2pcol_tiled tri_tiled tri 64 65536 float32 3 0
+prof tr2prow_tiled tri_tiled tri 64 65536 float32 2 0
 prof exec_bitonic_col exec_kernel exec_bitonic 64 1048576 float32 1 0
 prof exec_prefix_col exec_kernel exec_prefix 1024 1048576 float32 1 0
 prof exec_prefix_row exec_kernel exec_prefix 1024 1048576 float32 0 0
+prof exec_bitonic_col_jit bo_prog exec_bitonic 64 1048576 float32 1 1
+prof exec_bitonic_row_jit bo_prog exec_bitonic 64 1048576 float32 0 1
+prof exec_prefix_col_jit bo_prog exec_prefix 1024 1048576 float32 1 1
 # (compute-sanitizer was closed on the GPU pool late in round 2; the r02 sanitizer logs predate the
 #  cooperative column-wise preload)
 timeout 1200 python bench.py --sweep > $OUT/sweep.json 2> $OUT/sweep.err; echo "sweep rc=$?"
