@@ -111,7 +111,6 @@ __device__ __forceinline__ void cp_async4(void *dst, const void *src) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
-
 // S[u][v] = min(S[u][v], min_w A[u].w + B[w].v) for one 4-wide k chunk
 __device__ __forceinline__ float comp(const float4 &v, int i) { return i == 0 ? v.x : i == 1 ? v.y : i == 2 ? v.z : v.w; }
 __device__ __forceinline__ int comp(const int4 &v, int i) { return i == 0 ? v.x : i == 1 ? v.y : i == 2 ? v.z : v.w; }
@@ -741,7 +740,9 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
                 for (int j = KJ - 1; j >= 0; --j) {
                     const unsigned bal = __ballot_sync(0xffffffffu, a + 1 + li + LPI * j < b && r[j] == best) & own;
                     // a select, not a branch: measured 0.832 vs 0.866 ms for TR-2 + chords (a
-                    // select-only walk state machine below was slower again, 0.871)
+                    // select-only walk state machine below was slower again, 0.871; the min and
+                    // the k as two redux.sync over the instance's lanes -- CREDUX, serialised per
+                    // lane mask by WARPSYNC.EXCLUSIVE -- 0.887 against 0.834)
                     const int kj = a + 1 + ((__ffs(bal) - 1) >> (IPW == 4 ? 2 : IPW == 2 ? 1 : 0)) + LPI * j;
                     k = bal ? kj : k;
                 }
