@@ -742,7 +742,9 @@ tri_tiled_kernel(const T *__restrict__ c, T *__restrict__ out, int16_t *__restri
                     // a select, not a branch: measured 0.832 vs 0.866 ms for TR-2 + chords (a
                     // select-only walk state machine below was slower again, 0.871; the min and
                     // the k as two redux.sync over the instance's lanes -- CREDUX, serialised per
-                    // lane mask by WARPSYNC.EXCLUSIVE -- 0.887 against 0.834)
+                    // lane mask by WARPSYNC.EXCLUSIVE -- 0.887 against 0.834; warp-uniform
+                    // bounds that skip empty candidate groups, butterfly rounds and whole
+                    // triangle cells -- 0.982)
                     const int kj = a + 1 + ((__ffs(bal) - 1) >> (IPW == 4 ? 2 : IPW == 2 ? 1 : 0)) + LPI * j;
                     k = bal ? kj : k;
                 }
