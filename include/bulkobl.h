@@ -218,7 +218,8 @@ int bulk_program_release(int64_t handle);
 /*     coalesced load / store of the words read / written; larger: direct     */
 /*     loads grouped 32 at a time); row-wise msize <= 95 (rows staged through  */
 /*     shared memory).  BO_EUNSUPPORTED otherwise (row-wise msize > 95, more  */
-/*     than 200000 instructions) -- the interpreter keeps serving the call;   */
+/*     than 200000 instructions, libnvrtc.so.12 not found: it is dlopen'ed at */
+/*     the first compile, not linked) -- the interpreter keeps serving;       */
 /*     BO_ECUDA with the NVRTC log if compilation fails; BO_EINVAL on an      */
 /*     unknown handle or a packed layout.  Not while a stream is capturing.   */
 /*   bulk_program_source: the CUDA source bulk_program_compile builds (NUL-   */

@@ -75,10 +75,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
             sys.stderr.write(text)
     if failed:
         raise RuntimeError("nvcc failed")
-    # NVRTC (compiled programs, jit.cu) from the toolkit this image and the GPU boxes share
-    cuda_lib = os.path.join(os.path.dirname(os.path.dirname(os.path.realpath(NVCC))), "lib64")
-    subprocess.check_call([NVCC, *FLAGS, *objs, "-o", LIB, "-lrt", "-L" + cuda_lib, "-lnvrtc",
-                           "-Xlinker", "-rpath=" + cuda_lib])
+    subprocess.check_call([NVCC, *FLAGS, *objs, "-o", LIB, "-lrt", "-ldl"])   # (NVRTC: dlopen, jit.cu)
     return LIB
 
 

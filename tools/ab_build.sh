@@ -10,5 +10,5 @@ for f in paper_conf_ipps_tanitni14_b200/csrc/*.cu; do
   nvcc $F -c $f -o $out/$(basename $f).o & pids+=($!)
 done
 for p in ${pids[@]}; do wait $p; done
-nvcc -gencode arch=compute_100a,code=sm_100a -shared -cudart static $out/*.o -o $out/libbulkobl.so -lrt -L/usr/local/cuda/lib64 -lnvrtc -Xlinker -rpath=/usr/local/cuda/lib64
+nvcc -gencode arch=compute_100a,code=sm_100a -shared -cudart static $out/*.o -o $out/libbulkobl.so -lrt -ldl
 echo "built $out/libbulkobl.so"
