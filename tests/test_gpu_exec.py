@@ -300,6 +300,8 @@ def _compiled_case(kind, msize, t, seed, dt):
         return _fusable_program(msize, 6, t, seed)
     if kind == "bitonic":
         return programs.bitonic_sort(msize).array()
+    if kind == "opt":                                # Algorithm OPT written out (t = seed vertices)
+        return programs.optimal_triangulation(seed, dt).array()
     return programs.prefix_sums(msize, dt).array()
 
 
@@ -309,7 +311,9 @@ def _compiled_case(kind, msize, t, seed, dt):
                                                ("random", 96, 900, 24), ("random", 130, 1500, 25),
                                                ("random", 400, 1500, 26), ("fusable", 9, 600, 27),
                                                ("fusable", 300, 800, 28), ("bitonic", 64, 0, 0), ("bitonic", 1, 0, 0),
-                                               ("prefix", 33, 0, 0), ("prefix", 300, 0, 0)])
+                                               ("prefix", 33, 0, 0), ("prefix", 300, 0, 0),
+                                               ("opt", programs.optimal_triangulation(8).msize, 0, 8),
+                                               ("opt", programs.optimal_triangulation(12).msize, 0, 12)])
 def test_compiled_program_matches_oracle(dt, layout, kind, msize, t, seed):
     prog = _compiled_case(kind, msize, t, seed, dt)
     prep = bo.prepare(prog, msize)
