@@ -94,6 +94,9 @@ WORKLOADS = {
     "exec_bitonic_row_jit": dict(seed=6, algo="exec", prog="bitonic", n=64, p=2 ** 20, dtype="float32", layout=0,
                                  variant=0, jit=True,
                                  desc="NEXT-3: the bitonic sort program compiled, row-wise (rows staged in shared memory)"),
+    "exec_prefix_row_jit": dict(seed=2, algo="exec", prog="prefix", n=1024, p=2 ** 20, dtype="float32", layout=0,
+                                variant=0, jit=True,
+                                desc="NEXT-3: Algorithm Prefix-sums as a program, compiled (windowed rows), row-wise"),
     "exec_prefix_col_jit": dict(seed=2, algo="exec", prog="prefix", n=1024, p=2 ** 20, dtype="float32", layout=1,
                                 variant=0, jit=True,
                                 desc="NEXT-3: Algorithm Prefix-sums as a program, compiled (streaming shape), column-wise"),
@@ -120,7 +123,7 @@ WORKLOADS = {
 }
 EXTRAS = ["ps2col", "ps2tr", "tr_transpose", "ps1", "tr1", "tr1col", "tr1packed", "tr2", "tr2col", "tr2packed", "tr2chords", "tr512", "ps2naive_col", "ps2naive_row", "tr2umm",
           "exec_bitonic_col", "exec_bitonic_row", "exec_prefix_col", "exec_prefix_row",
-          "exec_bitonic_col_jit", "exec_bitonic_row_jit", "exec_prefix_col_jit",
+          "exec_bitonic_col_jit", "exec_bitonic_row_jit", "exec_prefix_col_jit", "exec_prefix_row_jit",
           "ps32k", "ps32k_col", "ps32k_naive_row", "ps32k_naive_col", "tr8", "tr8col", "tr8_umm_row", "tr8_umm_col"]
 # The paper's own fitted GTX Titan models, in ms for p instances: context for the
 # extras of the same shape, never a target (another machine, another decade)

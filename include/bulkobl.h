@@ -217,7 +217,9 @@ int bulk_program_release(int64_t handle);
 /*     Shapes: column-wise any msize (msize <= 128: memory in registers,      */
 /*     coalesced load / store of the words read / written; larger: direct     */
 /*     loads grouped 32 at a time); row-wise msize <= 95 (rows staged through  */
-/*     shared memory).  BO_EUNSUPPORTED otherwise (row-wise msize > 95, more  */
+/*     shared memory) or larger when the addresses stay in 64-word windows    */
+/*     (>= 8 accesses per window; each window staged through shared memory).  */
+/*     BO_EUNSUPPORTED otherwise (other row-wise programs, more               */
 /*     than 200000 instructions, libnvrtc.so.12 not found: it is dlopen'ed at */
 /*     the first compile, not linked) -- the interpreter keeps serving;       */
 /*     BO_ECUDA with the NVRTC log if compilation fails; BO_EINVAL on an      */

@@ -303,13 +303,18 @@ class Prepared:
         _check(lib().bulk_program_prepare(code.ctypes.data, self.t, self.msize, self.nregs, self.buf.data_ptr(),
                                           self.buf.numel(), _stream(stream, self.buf), ctypes.byref(h)))
         self.handle = h.value
+        # the upload is ordered on `stream` only: wait for it here (one-time setup), so the
+        # program may then run on any stream -- an execute on another stream could otherwise
+        # read the device program before its words arrive
+        (stream if stream is not None else torch.cuda.current_stream(self.buf.device)).synchronize()
 
     def compile(self, dtype=torch.float32, layout: int = COLUMN_WISE) -> bool:
         """Build the straight-line kernel of this program for (dtype, layout)
         (bulk_program_compile, NVRTC for sm_100a; host-blocking, cached).  True
         when later execute() calls with that dtype and layout run it; False when
-        the shape is not compiled (row-wise with msize > 95) and the
-        interpreter keeps serving them."""
+        the shape is not compiled (row-wise programs with msize > 95 whose
+        addresses do not stay in 64-word windows) and the interpreter keeps
+        serving them."""
         code = _DTYPES[dtype] if not isinstance(dtype, int) else dtype
         rc = lib().bulk_program_compile(self.handle, code, layout)
         if rc == -2:

@@ -23,8 +23,12 @@
 //             issued together ahead of the block (a LOAD of an address STOREd
 //             earlier in the block takes the stored value), so each thread keeps
 //             up to 32 loads in flight instead of one dependent load per step.
-// Row-wise programs with larger memories are not compiled (the interpreter's
-// windowed staging serves them).
+//   W-row     larger msize, row-wise: the program cut into segments whose
+//             addresses span <= 64 words; per segment the CTA's 128 rows' window
+//             is staged through shared memory (coalesced), the segment runs on it
+//             and it is written back if stored to -- when the windows are reused
+//             (>= 8 accesses per segment on average, <= 1024 segments); other
+//             row-wise programs are not compiled (the interpreter serves them).
 //
 // Semantics are the header's, instruction by instruction: registers start at
 // 0; int32 ADD / SUB wrap mod 2^32 (done in uint32); fp32 ADD / SUB are
@@ -39,6 +43,8 @@
 #include <dlfcn.h>
 #include <nvrtc.h>
 
+#include <algorithm>
+#include <climits>
 #include <functional>
 #include <map>
 #include <mutex>
@@ -62,11 +68,13 @@ constexpr int kJitThreads = 128;
 constexpr int kStreamGroup = BO_JIT_GROUP;        // LOADs issued ahead per block (streaming shape)
 constexpr int64_t kMaxJitInstructions = 200000;   // NVRTC time grows with the program (~1 s at 20K)
 
-enum Shape { kRegColumn, kRegRow, kStreamColumn, kNone };
+enum Shape { kRegColumn, kRegRow, kStreamColumn, kWinRow, kNone };
 
-Shape jit_shape(int64_t msize, int layout) {
+bool win_row_ok(const int32_t *prog, int64_t t);
+Shape jit_shape(const int32_t *prog, int64_t t, int64_t msize, int layout) {
     if (layout == BO_COLUMN_WISE) return msize <= 128 ? kRegColumn : kStreamColumn;
     if (layout == BO_ROW_WISE && msize <= 95) return kRegRow;   // 128 x 96 x 4 B = 48 KB static smem
+    if (layout == BO_ROW_WISE && win_row_ok(prog, t)) return kWinRow;
     return kNone;
 }
 
@@ -89,6 +97,46 @@ std::string op_expr(int32_t op, int32_t x, int32_t y, int32_t z, bool f32) {
     }
     s << ";\n";
     return s.str();
+}
+
+// Windowed row-wise shape: cut the program greedily into segments whose memory
+// addresses span <= kWin words.
+constexpr int kWin = 64;
+struct Segment {
+    int64_t i, e;
+    int32_t lo, len;
+    bool stores;
+};
+std::vector<Segment> win_segments(const int32_t *prog, int64_t t) {
+    std::vector<Segment> seg;
+    int64_t i = 0;
+    while (i < t) {
+        int64_t e = i;
+        int32_t lo = INT32_MAX, hi = -1;
+        bool stores = false;
+        for (; e < t; ++e) {
+            const int32_t op = prog[4 * e];
+            if (op != 0 && op != 1) continue;
+            const int32_t a = op == 0 ? prog[4 * e + 2] : prog[4 * e + 1];
+            const int32_t nlo = std::min(lo, a), nhi = std::max(hi, a);
+            if (nhi - nlo + 1 > kWin) break;
+            lo = nlo, hi = nhi;
+            stores |= op == 1;
+        }
+        if (hi < 0) lo = 0, hi = 0;                  // registers only
+        seg.push_back({i, e, lo, hi - lo + 1, stores});
+        i = e;
+    }
+    return seg;
+}
+// worth compiling only when the windows are reused: >= 8 memory accesses per segment on
+// average (the interpreter's windowing rule) and a bounded number of segments (each one
+// is two staged copies in the generated code)
+bool win_row_ok(const int32_t *prog, int64_t t) {
+    int64_t mem = 0;
+    for (int64_t i = 0; i < t; ++i) mem += prog[4 * i] == 0 || prog[4 * i] == 1;
+    const auto seg = win_segments(prog, t);
+    return seg.size() <= 1024 && mem >= 8 * static_cast<int64_t>(seg.size());
 }
 
 std::string generate(const int32_t *prog, int64_t t, int64_t msize, int nregs, int dtype, Shape shape) {
@@ -153,6 +201,39 @@ std::string generate(const int32_t *prog, int64_t t, int64_t msize, int nregs, i
                 s << "  __syncthreads();\n";
                 s << "  for (int i = threadIdx.x; i < cnt * " << msize << "; i += " << kJitThreads << ") { const int q = i / "
                   << msize << ", a = i - q * " << msize << "; g[i] = tile[q * " << msize + 1 << " + a]; }\n";
+            }
+        }
+    } else if (shape == kWinRow) {
+        // row-wise, larger memories: the program in segments whose addresses span <= kWin
+        // words; per segment the CTA's 128 rows' window [lo, lo+len) is staged through shared
+        // memory (coalesced: consecutive threads take consecutive words of a row), the
+        // segment runs on it, and it is written back when the segment stored into it
+        s << "  __shared__ T tile[" << kJitThreads * (kWin + 1) << "];\n";
+        s << "  const long long j0 = (long long)blockIdx.x * " << kJitThreads << ";\n";
+        s << "  const int cnt = (int)(p - j0 < " << kJitThreads << " ? p - j0 : " << kJitThreads << ");\n";
+        s << "  T *__restrict__ g = mem + j0 * " << msize << "LL;\n";
+        s << "  T *sr = tile + threadIdx.x * " << kWin + 1 << ";\n";
+        bool first_seg = true;
+        for (const Segment &g : win_segments(prog, t)) {
+            const int32_t lo = g.lo, len = g.len;
+            if (!first_seg) s << "  __syncthreads();\n";
+            first_seg = false;
+            s << "#pragma unroll 8\n  for (int i = threadIdx.x; i < cnt * " << len << "; i += " << kJitThreads
+              << ") { const int q = i / " << len << ", a = i - q * " << len << "; tile[q * " << kWin + 1
+              << " + a] = g[(long long)q * " << msize << "LL + " << lo << " + a]; }\n";
+            s << "  __syncthreads();\n  if (threadIdx.x < cnt) {\n";
+            for (int64_t k = g.i; k < g.e; ++k) {
+                const int32_t op = prog[4 * k], x = prog[4 * k + 1], y = prog[4 * k + 2], z = prog[4 * k + 3];
+                if (op == 0) s << "  r" << x << " = sr[" << y - lo << "];\n";
+                else if (op == 1) s << "  sr[" << x - lo << "] = r" << y << ";\n";
+                else s << "  " << op_expr(op, x, y, z, f32);
+            }
+            s << "  }\n";
+            if (g.stores) {
+                s << "  __syncthreads();\n";
+                s << "#pragma unroll 8\n  for (int i = threadIdx.x; i < cnt * " << len << "; i += " << kJitThreads
+                  << ") { const int q = i / " << len << ", a = i - q * " << len << "; g[(long long)q * " << msize
+                  << "LL + " << lo << " + a] = tile[q * " << kWin + 1 << " + a]; }\n";
             }
         }
     } else {   // kStreamColumn
@@ -286,8 +367,10 @@ int compile_source(const std::string &src, Compiled *out) {
 }  // namespace
 
 int jit_compile(const int32_t *prog, int64_t t, int64_t msize, int nregs, int dtype, int layout, JitKernel *out) {
-    const Shape shape = jit_shape(msize, layout);
-    if (shape == kNone) return fail(BO_EUNSUPPORTED, "program compile: row-wise programs need msize <= 95");
+    const Shape shape = jit_shape(prog, t, msize, layout);
+    if (shape == kNone)
+        return fail(BO_EUNSUPPORTED, "program compile: row-wise programs need msize <= 95 or addresses that stay "
+                                     "within 64-word windows (>= 8 accesses per window)");
     if (t > kMaxJitInstructions) return fail(BO_EUNSUPPORTED, "program compile: more than 200000 instructions");
     const std::string src = generate(prog, t, msize, nregs, dtype, shape);
     const size_t key = std::hash<std::string>{}(src);
@@ -323,7 +406,7 @@ int launch_jit(const JitKernel &k, void *mem, int64_t p, cudaStream_t st) {
 }
 
 std::string jit_source(const int32_t *prog, int64_t t, int64_t msize, int nregs, int dtype, int layout) {
-    const Shape shape = jit_shape(msize, layout);
+    const Shape shape = jit_shape(prog, t, msize, layout);
     return shape == kNone ? std::string() : generate(prog, t, msize, nregs, dtype, shape);
 }
 

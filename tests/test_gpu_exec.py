@@ -318,7 +318,12 @@ def test_compiled_program_matches_oracle(dt, layout, kind, msize, t, seed):
     prog = _compiled_case(kind, msize, t, seed, dt)
     prep = bo.prepare(prog, msize)
     compiled = prep.compile(getattr(torch, dt), layout)
-    assert compiled == (layout == bo.COLUMN_WISE or msize <= 95)
+    if layout == bo.COLUMN_WISE or msize <= 95:
+        assert compiled
+    elif kind in ("random", "opt"):                  # scattered addresses: no window reuse, not compiled
+        assert not compiled
+    else:                                            # row-wise windows: prefix / fusable programs
+        assert compiled
     if compiled:
         assert "bo_prog" in prep.source(getattr(torch, dt), layout)
     for p in (301, 128, 1):
