@@ -102,6 +102,9 @@ std::string op_expr(int32_t op, int32_t x, int32_t y, int32_t z, bool f32) {
 // Windowed row-wise shape: cut the program greedily into segments whose memory
 // addresses span <= kWin words.
 constexpr int kWin = 64;
+#ifndef BO_JIT_WIN_UNROLL
+#define BO_JIT_WIN_UNROLL 8   // window copies (prefix program row-wise): 8 1.82, 16 1.90, 32 2.59, 64 6.23 ms
+#endif
 struct Segment {
     int64_t i, e;
     int32_t lo, len;
@@ -218,7 +221,7 @@ std::string generate(const int32_t *prog, int64_t t, int64_t msize, int nregs, i
             const int32_t lo = g.lo, len = g.len;
             if (!first_seg) s << "  __syncthreads();\n";
             first_seg = false;
-            s << "#pragma unroll 8\n  for (int i = threadIdx.x; i < cnt * " << len << "; i += " << kJitThreads
+            s << "#pragma unroll " << BO_JIT_WIN_UNROLL << "\n  for (int i = threadIdx.x; i < cnt * " << len << "; i += " << kJitThreads
               << ") { const int q = i / " << len << ", a = i - q * " << len << "; tile[q * " << kWin + 1
               << " + a] = g[(long long)q * " << msize << "LL + " << lo << " + a]; }\n";
             s << "  __syncthreads();\n  if (threadIdx.x < cnt) {\n";
@@ -231,7 +234,7 @@ std::string generate(const int32_t *prog, int64_t t, int64_t msize, int nregs, i
             s << "  }\n";
             if (g.stores) {
                 s << "  __syncthreads();\n";
-                s << "#pragma unroll 8\n  for (int i = threadIdx.x; i < cnt * " << len << "; i += " << kJitThreads
+                s << "#pragma unroll " << BO_JIT_WIN_UNROLL << "\n  for (int i = threadIdx.x; i < cnt * " << len << "; i += " << kJitThreads
                   << ") { const int q = i / " << len << ", a = i - q * " << len << "; g[(long long)q * " << msize
                   << "LL + " << lo << " + a] = tile[q * " << kWin + 1 << " + a]; }\n";
             }
