@@ -230,6 +230,11 @@ int bulk_program_release(int64_t handle);
 /* ------------------------------------------------------------------------- */
 int bulk_program_compile(int64_t handle, int dtype, int layout);
 int bulk_program_source(int64_t handle, int dtype, int layout, char *buf, size_t cap, size_t *len);
+/*   bulk_program_generate: the same source for a HOST program (prog/t/msize/ */
+/*     nregs validated as bulk_execute); no device, no handle -- for           */
+/*     inspecting the generated kernel on a machine without a GPU.            */
+int bulk_program_generate(const int32_t *prog, int64_t t, int64_t msize, int nregs, int dtype, int layout, char *buf,
+                          size_t cap, size_t *len);
 
 /* ------------------------------------------------------------------------- */
 /* Layout transpose (row-wise <-> column-wise arrangement):        */

@@ -69,6 +69,7 @@ def lib() -> ctypes.CDLL:
             "bulk_execute_prepared": ([i64, vp, i64, i64, i32, i32, vp], i32),
             "bulk_program_compile": ([i64, i32, i32], i32),
             "bulk_program_source": ([i64, i32, i32, vp, sz, ctypes.POINTER(sz)], i32),
+            "bulk_program_generate": ([vp, i64, i64, i32, i32, i32, vp, sz, ctypes.POINTER(sz)], i32),
             "bulk_program_release": ([i64], i32),
             "bulk_prefix_sums_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
             "bulk_triangulation_host": ([vp, vp, i64, i64, i32, i32, i32, vp, sz, vp], i32),
@@ -335,6 +336,20 @@ class Prepared:
         if getattr(self, "handle", 0) and _lib is not None:
             _lib.bulk_program_release(self.handle)
             self.handle = 0
+
+
+def program_source(program, msize: int, dtype=torch.float32, layout: int = COLUMN_WISE) -> str:
+    """The CUDA source bulk_program_compile would build for `program` on
+    `msize`-word memories (bulk_program_generate: host only, no GPU needed)."""
+    code, nregs = _program_code(program)
+    d = _DTYPES[dtype] if not isinstance(dtype, int) else dtype
+    n = ctypes.c_size_t(0)
+    _check(lib().bulk_program_generate(code.ctypes.data, code.shape[0], int(msize), nregs, d, layout, None, 0,
+                                       ctypes.byref(n)))
+    buf = ctypes.create_string_buffer(n.value)
+    _check(lib().bulk_program_generate(code.ctypes.data, code.shape[0], int(msize), nregs, d, layout, buf, n.value,
+                                       ctypes.byref(n)))
+    return buf.value.decode()
 
 
 def prepare(program, msize: int, device="cuda", stream=None) -> Prepared:

@@ -529,6 +529,22 @@ int bulk_program_source(int64_t handle, int dtype, int layout, char *buf, size_t
     return BO_OK;
 }
 
+int bulk_program_generate(const int32_t *prog, int64_t t, int64_t msize, int nregs, int dtype, int layout, char *buf,
+                          size_t cap, size_t *len) {
+    t_err.clear();
+    if (!len) return fail(BO_EINVAL, "program generate: NULL len");
+    if (int rc = exec_check_sizes(t, msize, 0, nregs)) return rc;
+    if (t > 0 && !prog) return fail(BO_EINVAL, "program generate: NULL program");
+    if (!valid_dtype(dtype)) return fail(BO_EINVAL, "program generate: bad dtype");
+    bool uninit_read = false;
+    if (int rc = exec_validate(prog, t, msize, nregs, &uninit_read)) return rc;
+    const std::string s = jit_source(prog, t, msize, nregs, dtype, layout);
+    if (s.empty()) return fail(BO_EUNSUPPORTED, "program generate: this arrangement is not compiled");
+    *len = s.size() + 1;
+    if (buf && cap >= s.size() + 1) std::memcpy(buf, s.c_str(), s.size() + 1);
+    return BO_OK;
+}
+
 int bulk_triangulation_chords(const void *c, void *out, int16_t *chords, int64_t n, int64_t p, int dtype,
                               int layout, void *stream) {
     t_err.clear();
