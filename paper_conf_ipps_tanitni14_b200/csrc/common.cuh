@@ -89,6 +89,14 @@ inline bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
+// The first A-byte aligned address of a dynamic shared-memory buffer, as an
+// offset from it: a pointer rebuilt from an integer loses the shared address
+// space, and the compiler then emits generic LD / ST for every access (and
+// cannot reorder them) -- measured in ps_fused_row_tma's scan.
+template <int A>
+__device__ __forceinline__ uint8_t *smem_align(uint8_t *raw) {
+    return raw + ((A - (smem_u32(raw) & (A - 1))) & (A - 1));
+}
 
 __device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));

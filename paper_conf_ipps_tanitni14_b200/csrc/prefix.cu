@@ -138,8 +138,7 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
     constexpr uint32_t kBoxBytes = fr::Cfg<kInst>::kBoxBytes;
     constexpr uint32_t kStageBytes = fr::Cfg<kInst>::kStageBytes;
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                               ~uintptr_t(1023));
+    uint8_t *buf = smem_align<1024>(smem_raw);
     uint64_t *full = reinterpret_cast<uint64_t *>(buf + kStages * kStageBytes);
     int *stage_tile = reinterpret_cast<int *>(full + kStages);    // tile of each ring slot, -1 = end
     int *stage_chunk = stage_tile + kStages;                      // its first chunk
@@ -199,20 +198,37 @@ ps_fused_row_tma(const __grid_constant__ CUtensorMap src_map, const __grid_const
         const int chunk = stage_chunk[s];
         const int cnt = kCps == 1 ? 1 : stage_cnt[s];
         if (chunk == 0) r = T(0);                       // new tile: r_j <- 0
+        // a box's 8 row pieces read into registers before the dependent chain, the next
+        // box's while this one is scanned (the swizzled addresses defeat the compiler's
+        // alias analysis, so in-place load / add / store pieces serialise on each other):
+        // with shared-space addressing, n = 32K p = 8K 0.468 -> 0.403 ms, n = 1024 p = 4096
+        // 17.9 -> 12.9 us, n = 4096 p = 8192 63 -> 55 us; PS-2 1.320 -> 1.318 ms
+        uint4 cur[kElems / 4], nxt[kElems / 4];
+#pragma unroll
+        for (int k = 0; k < kElems / 4; ++k)
+            cur[k] = *reinterpret_cast<const uint4 *>(buf + s * kStageBytes + swz128(tid, k));
 #pragma unroll
         for (int b = 0; b < kCps; ++b) {
             if (kCps > 1 && b >= cnt) break;
             uint8_t *box = buf + s * kStageBytes + b * kBoxBytes;
+            if (b + 1 < kCps && b + 1 < cnt) {
+#pragma unroll
+                for (int k = 0; k < kElems / 4; ++k)
+                    nxt[k] = *reinterpret_cast<const uint4 *>(box + kBoxBytes + swz128(tid, k));
+            }
 #pragma unroll
             for (int k = 0; k < kElems / 4; ++k) {
-                uint4 *q = reinterpret_cast<uint4 *>(box + swz128(tid, k));
-                uint4 v = *q;
+                uint4 v = cur[k];
                 r = add_wrap(r, bits_as<T>(v.x)); v.x = as_bits(r);   // r <- r + b[i]; b[i] <- r
                 r = add_wrap(r, bits_as<T>(v.y)); v.y = as_bits(r);
                 r = add_wrap(r, bits_as<T>(v.z)); v.z = as_bits(r);
                 r = add_wrap(r, bits_as<T>(v.w)); v.w = as_bits(r);
-                *q = v;
+                cur[k] = v;
             }
+#pragma unroll
+            for (int k = 0; k < kElems / 4; ++k) *reinterpret_cast<uint4 *>(box + swz128(tid, k)) = cur[k];
+#pragma unroll
+            for (int k = 0; k < kElems / 4; ++k) cur[k] = nxt[k];
         }
         fence_proxy_async_smem();
         __syncthreads();
@@ -270,8 +286,10 @@ ps_across_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant
     constexpr int kStages = ac::Cfg<kInst>::kStages;
     constexpr uint32_t kBoxBytes = ac::Cfg<kInst>::kBoxBytes;
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                               ~uintptr_t(1023));
+    // (a generic pointer on purpose: with shared-space accesses (smem_align) the scan
+    // loop schedules differently -- n = 32K p = 8K 0.382 -> 0.421 ms, though n = 1024
+    // p = 16384 gains 29.5 -> 23.8 us; batched register staging changes neither)
+    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     uint64_t *full = reinterpret_cast<uint64_t *>(buf + kStages * kBoxBytes);
     int *stage_tile = reinterpret_cast<int *>(full + kStages);
     int *stage_chunk = stage_tile + kStages;

@@ -38,8 +38,7 @@ transpose_tma_kernel(const __grid_constant__ CUtensorMap src_map,
     pdl_begin();
     using namespace tr;
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *base = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                                ~uintptr_t(1023));
+    uint8_t *base = smem_align<1024>(smem_raw);
     uint8_t *in_buf = base;                                   // kStages boxes
     uint8_t *out_buf = base + kStages * kBoxBytes;            // kOut boxes (2 sub-tiles each)
     uint64_t *full = reinterpret_cast<uint64_t *>(out_buf + kOut * kBoxBytes);

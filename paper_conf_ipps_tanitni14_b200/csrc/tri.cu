@@ -117,7 +117,7 @@ tri_thread_reg_tma(const __grid_constant__ CUtensorMap cmap, T *__restrict__ out
     // still holds, so one full barrier per slot and its phase parity suffice
     static_assert(S % W == 0 && S / W >= 1, "each warp owns S / W ring slots");
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t *buf = smem_align<1024>(smem_raw);
     uint64_t *bar = reinterpret_cast<uint64_t *>(buf + S * kBatchBytes);
     const int t = threadIdx.x & 31, warp = threadIdx.x >> 5;
     auto issue = [&](long long i) {                  // batch i of this CTA -> ring slot i % S
@@ -205,7 +205,7 @@ tri_thread_reg_packed(const T *__restrict__ c, T *__restrict__ out, long long p,
     constexpr int K = (N - 1) * (N - 2) / 2;
     constexpr uint32_t kBatchBytes = 32u * K * sizeof(T);
     extern __shared__ uint8_t smem_raw[];
-    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 127) & ~uintptr_t(127));
+    uint8_t *buf = smem_align<128>(smem_raw);
     uint64_t *bar = reinterpret_cast<uint64_t *>(buf + 2 * ((kBatchBytes + 127) & ~127u));
     const uint32_t stride = (kBatchBytes + 127) & ~127u;
     const int t = threadIdx.x;
