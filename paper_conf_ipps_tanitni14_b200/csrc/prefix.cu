@@ -110,12 +110,16 @@ template <int INST> struct Cfg {
     // (stages x chunks): 3 x 4 against 8 x 1 -- n = 32K p = 8K 0.477 vs 0.554 ms,
     // n = 4096 p = 8192 65 vs 73 us, n = 1024 p = 4096 18.2 vs 20.9 us, p = 32768 48.7
     // vs 50.5 us, p = 16384 23.9 vs 23.6 us; 4 x 4 and 6 x 4 lose at p = 16384 (34 us:
-    // fewer CTAs per SM than tiles), a 24 x 1 ring loses everywhere.
+    // fewer CTAs per SM than tiles), a 24 x 1 ring loses everywhere.  After the scan
+    // was register-staged (late round 2) the ring depth matters again: 6 x 2 (the same
+    // 48 KB) against 3 x 4 -- n = 32K p = 8K 0.369 vs 0.403 ms, n = 4096 p = 8192 48.2 vs
+    // 54.6 us, n = 1024 p = 16384 / 32768 22.1 / 45.6 vs 22.2 / 46.2 us, n = 1024
+    // p = 4096 13.3 vs 12.9 us; 4 x 4 loses at p = 16384 (26.9 us).
 #ifndef BO_FR_STAGES32
-#define BO_FR_STAGES32 3
+#define BO_FR_STAGES32 6
 #endif
 #ifndef BO_FR_CPS32
-#define BO_FR_CPS32 4
+#define BO_FR_CPS32 2
 #endif
     static constexpr int kStages = INST == 128 ? BO_FR_STAGES : BO_FR_STAGES32;
     static constexpr int kCps = INST == 128 ? 1 : BO_FR_CPS32;
