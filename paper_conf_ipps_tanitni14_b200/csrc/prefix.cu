@@ -270,8 +270,12 @@ namespace ac {
 // 32 x 8 1.356, 32 x 4 1.360, 64 x 3 1.356, 16 x 8 1.360
 constexpr int kElems = BO_AC_ROWS;          // rows per box
 constexpr int kStages = BO_AC_STAGES;
+// 32-instance blocks, ring depth with shared-space scan accesses (late round 2; the
+// round-2 generic pointer had 12): 4 / 6 / 8 / 12 / 24 stages -- n = 32K p = 8K 0.392 /
+// 0.358 / 0.401 / 0.425 / 0.535 ms, n = 4096 p = 8192 52.0 / 43.9 / 49.7 / 53.1 / 72.2 us
+// (generic, 12: 0.383 ms, 52.4 us), n = 1024 p = 16384 22.1 / 22.7 / 24.4 / 23.6 us (29.4)
 #ifndef BO_AC_STAGES32
-#define BO_AC_STAGES32 12
+#define BO_AC_STAGES32 6
 #endif
 template <int INST> struct Cfg {
     // 32-instance column blocks (small p, long columns): a deeper ring per CTA
@@ -290,10 +294,7 @@ ps_across_tma(const __grid_constant__ CUtensorMap src_map, const __grid_constant
     constexpr int kStages = ac::Cfg<kInst>::kStages;
     constexpr uint32_t kBoxBytes = ac::Cfg<kInst>::kBoxBytes;
     extern __shared__ uint8_t smem_raw[];
-    // (a generic pointer on purpose: with shared-space accesses (smem_align) the scan
-    // loop schedules differently -- n = 32K p = 8K 0.382 -> 0.421 ms, though n = 1024
-    // p = 16384 gains 29.5 -> 23.8 us; batched register staging changes neither)
-    uint8_t *buf = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t *buf = smem_align<1024>(smem_raw);
     uint64_t *full = reinterpret_cast<uint64_t *>(buf + kStages * kBoxBytes);
     int *stage_tile = reinterpret_cast<int *>(full + kStages);
     int *stage_chunk = stage_tile + kStages;
